@@ -1,0 +1,165 @@
+/*
+ * psb.h — C ABI of libpsb.so: exact k-nearest-neighbour queries by Parallel Scan
+ * and Backtrack (PSB) over a bulk-loaded n-ary R-tree, on NVIDIA B200 (sm_100a).
+ *
+ * Paper: M. Nam, J. Kim, B. Nam, "Parallel Tree Traversal for Nearest Neighbor
+ * Query on the GPU", ICPP 2016. Citations "P:Lx-y" are lines of that paper's text
+ * with the section / algorithm they fall in.
+ *
+ * Problem (§I; Alg. 1 "SearchKNN(Point Q, int k)" P:L403-405): given n
+ * points in d dimensions and a query point Q, return the k points closest to Q,
+ * exactly (§I, §VI).
+ *
+ * Conventions shared by every entry point (DESIGN.md §2 "Readings"):
+ *  - Distances are SQUARED Euclidean in binary32, accumulated over dimensions
+ *    0..d-1 in order, each subtraction, product and sum rounded to nearest-even
+ *    separately (no FMA, no flush-to-zero):
+ *        s = +0; for j: t = p[j] - q[j]; s = s + t*t.
+ *  - A result row holds the k smallest (dist, id) pairs under lexicographic order
+ *    (distance first, then id), ascending. If k > n the row is padded with
+ *    (id -1, dist +inf).
+ *  - Ids are 0-based input row numbers plus the index's id_base.
+ *  - Layouts: points[n][d], queries[q][d] fp32 row-major; out_ids[q][k] int32,
+ *    out_dists[q][k] fp32, row-major.
+ *  - Pointers to queries/outputs are CUDA device pointers on the index's device
+ *    (psb_build: points may be host or device memory).
+ *  - Query calls are asynchronous on `stream` (a cudaStream_t; NULL = legacy
+ *    default stream). Argument errors are returned synchronously without
+ *    launching; launch failures return PSB_ECUDA; errors during execution surface
+ *    at the caller's next synchronisation. Inputs must stay alive and unmodified
+ *    until the stream reaches the work.
+ *  - No entry point prints, aborts or throws. psb_last_error() returns a
+ *    thread-local message describing the last failure on the calling thread.
+ *  - An index is immutable after build: concurrent queries on different streams
+ *    are safe. It is bound to the device that was current at build time.
+ */
+#ifndef PSB_H
+#define PSB_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct psb_index psb_index; /* opaque */
+
+enum {
+    PSB_OK = 0,
+    PSB_EINVAL = -1,          /* bad argument (null pointer, range, non-finite coordinate) */
+    PSB_ENOMEM = -2,          /* host or device allocation failed                          */
+    PSB_ECUDA = -3,           /* CUDA runtime error (message in psb_last_error)           */
+    PSB_EUNSUPPORTED = -4     /* valid but outside this build (e.g. k > PSB_KMAX)         */
+};
+
+/* Leaf packing order for psb_build_ex `flags` (§IV-A: sort points by
+ * a space-filling-curve key and pack them into full leaves, bottom-up). */
+enum { PSB_PACK_HILBERT = 0, PSB_PACK_STR = 1 };
+
+#define PSB_KMAX 128          /* largest k served by the warp top-k (4 keys per lane) */
+#define PSB_DMAX 64           /* largest dimensionality                               */
+
+/* Bulk-load an R-tree over points[n][d] (§IV, bottom-up construction,
+ * with minimum bounding rectangles as the bounding shape, §I):
+ *  - points are ordered by a Hilbert key and packed left to right
+ *    into leaves of exactly `fanout` points (100% utilisation, P:L162-163,
+ *    P:L678-684); only the last leaf may be partial;
+ *  - every internal node has up to `fanout` children; each node stores its
+ *    children's MBRs as structure-of-arrays rows lo[d][fanout], hi[d][fanout]
+ *    (§V-A: "stored in SoA so that memory coalescing can be employed");
+ *  - leaves are contiguous in left-to-right order with sequence ids 0..L-1; the
+ *    parent of node i is i/fanout one level up and the right sibling of leaf j
+ *    is j+1 (the parent links and rightSibling of Alg. 1).
+ * `points` may be host or device memory; it is copied (the caller may free it
+ * afterwards). n >= 1, 1 <= d <= PSB_DMAX, fanout in {32,64,128,256,512}, all
+ * coordinates finite. Synchronous. Returns NULL on error (see psb_last_error). */
+psb_index *psb_build(const float *points, int64_t n, int32_t d, int32_t fanout);
+
+/* As psb_build, plus: returned ids are id_base + input row (data-sharded use:
+ * a shard over rows [r0, r1) of a global set passes id_base = r0;
+ * id_base >= 0 and id_base + n <= 2^31 - 1), and `flags` selects the packing
+ * (PSB_PACK_HILBERT or PSB_PACK_STR). On success *out receives the index. */
+int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int64_t id_base,
+                 uint32_t flags, psb_index **out);
+
+/* PSB kNN (Alg. 1, §III, with the readings of DESIGN.md §2): for each
+ * of the q queries, one warp descends greedily to the closest leaf to obtain an
+ * initial pruning distance (Alg. 1 l.3), then restarts at the root, descends to
+ * the leftmost child within the pruning distance whose leaves are not yet
+ * visited (l.16-26), scans leaves left to right while they improve the kNN set
+ * (l.32-41) and backtracks through parent links otherwise (l.27-30, l.42-45).
+ * 1 <= k <= PSB_KMAX (else PSB_EUNSUPPORTED), q >= 0 (q = 0 is a no-op). */
+int psb_knn(const psb_index *idx, const float *queries, int64_t q, int32_t k,
+            int32_t *out_ids, float *out_dists, void *stream);
+
+/* The paper's comparison algorithm: classic branch-and-bound kNN (Roussopoulos
+ * et al. [17], §III) run data-parallel on the GPU with parent links
+ * instead of a stack (§IV-D): children in (MINDIST, index) order,
+ * each leaf followed by a return to its parent. Same arguments and results as
+ * psb_knn. */
+int psb_knn_branch_and_bound(const psb_index *idx, const float *queries, int64_t q, int32_t k,
+                             int32_t *out_ids, float *out_dists, void *stream);
+
+/* GPU brute-force exhaustive kNN (the paper's other baseline, §I,
+ * P:L936-947 §V-D): every point against every query, same distance formula and
+ * order. Same arguments and results as psb_knn. May allocate stream-ordered
+ * scratch on `stream`. */
+int psb_knn_bruteforce(const psb_index *idx, const float *queries, int64_t q, int32_t k,
+                       int32_t *out_ids, float *out_dists, void *stream);
+
+/* Variant selector for the two tree traversals (measurement and ablations):
+ * bit 0 PSB_VAR_NOCACHE  — re-fetch every node on return instead of reusing the
+ *                          per-level MINDIST path cache (the paper's parent-link
+ *                          behaviour);
+ * bit 1 PSB_VAR_NOMAXDIST — skip the k-th-MAXDIST bound (Alg. 1 l.13-15).
+ * Results are identical for every variant. */
+enum { PSB_VAR_NOCACHE = 1, PSB_VAR_NOMAXDIST = 2 };
+int psb_knn_ex(const psb_index *idx, const float *queries, int64_t q, int32_t k,
+               int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant);
+enum { PSB_ALGO_PSB = 0, PSB_ALGO_BNB = 1, PSB_ALGO_BRUTE = 2 };
+
+/* Merge `parts` per-shard result sets ids/dists[parts][q][k] (each row ascending
+ * by (dist, id), ids global) into the first k of their union, out[q][k]
+ * (data-sharded mode: the step after the all-gather). Device pointers,
+ * asynchronous on `stream`. 1 <= parts, 1 <= k <= PSB_KMAX. */
+int psb_merge_topk(const int32_t *ids, const float *dists, int32_t parts, int64_t q, int32_t k,
+                   int32_t *out_ids, float *out_dists, void *stream);
+
+/* Shape of an index. Any output pointer may be NULL. `levels` counts internal
+ * levels (root at level `levels`, leaves at level 0); device_bytes is the index's
+ * device footprint. */
+int psb_index_info(const psb_index *idx, int64_t *n, int32_t *d, int32_t *fanout, int64_t *leaves,
+                   int32_t *levels, int64_t *device_bytes);
+
+/* Copy the index's flat arrays to host memory (tests, replicas). Layout of the
+ * exported blob (all little-endian):
+ *   int64 header[8] = {n, d, fanout, leaves L, levels H, id_base, total_nodes, 0}
+ *   int64 nodes_per_level[H+1]            (level 0 = L leaves)
+ *   float pts[L][d][fanout]               (leaf-blocked SoA; pad slots +inf)
+ *   int32 ids[L][fanout]                  (pad slots -1)
+ *   float nodes: for level 1..H, nodes_per_level[l] blocks of [d][2][fanout]
+ *                (row 2j = lo of dim j, row 2j+1 = hi; empty slots lo=+inf, hi=-inf)
+ * If host_buf is NULL or cap is too small, only *used is written (required size)
+ * and PSB_EINVAL is returned when host_buf is non-NULL. Synchronous. */
+int psb_index_export(const psb_index *idx, void *host_buf, int64_t cap, int64_t *used);
+
+/* Host-only bulk load (no CUDA call, no device needed): runs the same packing as
+ * psb_build_ex and writes the psb_index_export blob for it into host_buf
+ * (same size protocol as psb_index_export). For layout tests on machines without
+ * a GPU; a device index built from the same arguments exports identical bytes. */
+int psb_build_host_blob(const float *points, int64_t n, int32_t d, int32_t fanout, int64_t id_base,
+                        uint32_t flags, void *host_buf, int64_t cap, int64_t *used);
+
+/* Release the index and its device memory. NULL is a no-op. */
+void psb_free(psb_index *idx);
+
+/* Thread-local message for the last failing call on this thread ("" if none). */
+const char *psb_last_error(void);
+
+/* Library version string ("psb-b200 <version> sm_100a"). */
+const char *psb_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PSB_H */

@@ -1,0 +1,269 @@
+"""psb-b200 — exact kNN by Parallel Scan and Backtrack on NVIDIA B200 (sm_100a).
+
+Thin Python binding over ``libpsb.so`` (C ABI in ``include/psb.h``). Every step
+of the query path runs in the library's CUDA kernels; this module only marshals
+arguments: torch tensors provide device memory and streams. There is no CPU
+fallback: importing the package fails if ``libpsb.so`` has not been built
+(``python -c "import __graft_entry__ as g; g.build()"``).
+
+Names mirror the C ABI: ``psb_build``, ``psb_build_ex``, ``psb_knn``,
+``psb_knn_branch_and_bound``, ``psb_knn_bruteforce``, ``psb_knn_ex``,
+``psb_merge_topk``, ``psb_index_info``, ``psb_index_export``,
+``psb_build_host_blob``, ``psb_free``, ``psb_last_error``, ``psb_version``.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libpsb.so")
+
+PSB_OK, PSB_EINVAL, PSB_ENOMEM, PSB_ECUDA, PSB_EUNSUPPORTED = 0, -1, -2, -3, -4
+PSB_PACK_HILBERT, PSB_PACK_STR = 0, 1
+PSB_ALGO_PSB, PSB_ALGO_BNB, PSB_ALGO_BRUTE = 0, 1, 2
+PSB_VAR_NOCACHE, PSB_VAR_NOMAXDIST = 1, 2
+PSB_KMAX, PSB_DMAX = 128, 64
+FANOUTS = (32, 64, 128, 256, 512)
+
+# every symbol include/psb.h declares (tests check the .so exports all of them)
+EXPORTS = ("psb_build", "psb_build_ex", "psb_knn", "psb_knn_branch_and_bound", "psb_knn_bruteforce",
+           "psb_knn_ex", "psb_merge_topk", "psb_index_info", "psb_index_export", "psb_build_host_blob",
+           "psb_free", "psb_last_error", "psb_version")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"libpsb.so not built at {LIB_PATH}: run __graft_entry__.build() "
+                      "(there is no CPU fallback)")
+
+_lib = ctypes.CDLL(LIB_PATH)
+_vp, _i64, _i32, _u32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint32
+_P = ctypes.POINTER
+_sig = {
+    "psb_build": (_vp, [_vp, _i64, _i32, _i32]),
+    "psb_build_ex": (ctypes.c_int, [_vp, _i64, _i32, _i32, _i64, _u32, _P(_vp)]),
+    "psb_knn": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp]),
+    "psb_knn_branch_and_bound": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp]),
+    "psb_knn_bruteforce": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp]),
+    "psb_knn_ex": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp, _i32, _u32]),
+    "psb_merge_topk": (ctypes.c_int, [_vp, _vp, _i32, _i64, _i32, _vp, _vp, _vp]),
+    "psb_index_info": (ctypes.c_int, [_vp, _P(_i64), _P(_i32), _P(_i32), _P(_i64), _P(_i32), _P(_i64)]),
+    "psb_index_export": (ctypes.c_int, [_vp, _vp, _i64, _P(_i64)]),
+    "psb_build_host_blob": (ctypes.c_int, [_vp, _i64, _i32, _i32, _i64, _u32, _vp, _i64, _P(_i64)]),
+    "psb_free": (None, [_vp]),
+    "psb_last_error": (ctypes.c_char_p, []),
+    "psb_version": (ctypes.c_char_p, []),
+}
+for _name, (_res, _args) in _sig.items():
+    _f = getattr(_lib, _name)
+    _f.restype, _f.argtypes = _res, _args
+
+
+class PSBError(RuntimeError):
+    def __init__(self, code: int, where: str):
+        self.code = code
+        super().__init__(f"{where} failed ({code}): {psb_last_error()}")
+
+
+def _check(rc: int, where: str):
+    if rc != PSB_OK:
+        raise PSBError(rc, where)
+
+
+def psb_last_error() -> str:
+    return _lib.psb_last_error().decode()
+
+
+def psb_version() -> str:
+    return _lib.psb_version().decode()
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def _stream_handle(stream) -> int:
+    torch = _torch()
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return int(stream.cuda_stream) if hasattr(stream, "cuda_stream") else int(stream)
+
+
+class Index:
+    """Owns a psb_index* (device memory on the device current at build time)."""
+
+    def __init__(self, handle: int):
+        self._h = ctypes.c_void_p(handle)
+        n, d, f, L, H, b = _i64(), _i32(), _i32(), _i64(), _i32(), _i64()
+        _check(_lib.psb_index_info(self._h, ctypes.byref(n), ctypes.byref(d), ctypes.byref(f),
+                                   ctypes.byref(L), ctypes.byref(H), ctypes.byref(b)), "psb_index_info")
+        self.n, self.d, self.fanout = n.value, d.value, f.value
+        self.leaves, self.levels, self.device_bytes = L.value, H.value, b.value
+        self.device = _torch().cuda.current_device()
+
+    @property
+    def handle(self):
+        return self._h
+
+    def free(self):
+        if self._h is not None and self._h.value:
+            _lib.psb_free(self._h)
+        self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+    def info(self) -> dict:
+        return {"n": self.n, "d": self.d, "fanout": self.fanout, "leaves": self.leaves,
+                "levels": self.levels, "device_bytes": self.device_bytes}
+
+
+def _as_points(points):
+    """Host numpy / CPU tensor / CUDA tensor -> (pointer, keepalive, n, d)."""
+    torch = _torch()
+    if isinstance(points, np.ndarray):
+        a = np.ascontiguousarray(points, dtype=np.float32)
+        return a.ctypes.data, a, a.shape[0], a.shape[1]
+    t = points.contiguous()
+    if t.dtype != torch.float32:
+        raise TypeError("points must be float32")
+    return t.data_ptr(), t, t.shape[0], t.shape[1]
+
+
+def psb_build_ex(points, fanout: int, id_base: int = 0, packing: int = PSB_PACK_HILBERT) -> Index:
+    """Bulk-load the R-tree (include/psb.h psb_build_ex) on the current CUDA device."""
+    ptr, keep, n, d = _as_points(points)
+    out = ctypes.c_void_p()
+    _check(_lib.psb_build_ex(ptr, n, d, fanout, id_base, packing, ctypes.byref(out)), "psb_build_ex")
+    del keep
+    return Index(out.value)
+
+
+def psb_build(points, fanout: int) -> Index:
+    ptr, keep, n, d = _as_points(points)
+    h = _lib.psb_build(ptr, n, d, fanout)
+    if not h:
+        raise PSBError(PSB_EINVAL, "psb_build")
+    return Index(h)
+
+
+def _query_buffers(index: Index, queries, k: int, out):
+    torch = _torch()
+    if not (queries.is_cuda and queries.dtype == torch.float32 and queries.dim() == 2
+            and queries.shape[1] == index.d):
+        raise ValueError(f"queries must be a CUDA float32 [q, {index.d}] tensor")
+    queries = queries.contiguous()
+    q = queries.shape[0]
+    if out is None:
+        ids = torch.empty((q, k), dtype=torch.int32, device=queries.device)
+        dists = torch.empty((q, k), dtype=torch.float32, device=queries.device)
+    else:
+        ids, dists = out
+    return queries, q, ids, dists
+
+
+def psb_knn_ex(index: Index, queries, k: int, algo: int = PSB_ALGO_PSB, variant: int = 0,
+               stream=None, out=None):
+    """Asynchronous on `stream` (default: torch's current stream). Returns (ids, dists)."""
+    queries, q, ids, dists = _query_buffers(index, queries, k, out)
+    _check(_lib.psb_knn_ex(index.handle, queries.data_ptr(), q, k, ids.data_ptr(), dists.data_ptr(),
+                           _stream_handle(stream), algo, variant), "psb_knn_ex")
+    return ids, dists
+
+
+def psb_knn(index: Index, queries, k: int, stream=None, out=None):
+    queries, q, ids, dists = _query_buffers(index, queries, k, out)
+    _check(_lib.psb_knn(index.handle, queries.data_ptr(), q, k, ids.data_ptr(), dists.data_ptr(),
+                        _stream_handle(stream)), "psb_knn")
+    return ids, dists
+
+
+def psb_knn_branch_and_bound(index: Index, queries, k: int, stream=None, out=None):
+    queries, q, ids, dists = _query_buffers(index, queries, k, out)
+    _check(_lib.psb_knn_branch_and_bound(index.handle, queries.data_ptr(), q, k, ids.data_ptr(),
+                                         dists.data_ptr(), _stream_handle(stream)),
+           "psb_knn_branch_and_bound")
+    return ids, dists
+
+
+def psb_knn_bruteforce(index: Index, queries, k: int, stream=None, out=None):
+    queries, q, ids, dists = _query_buffers(index, queries, k, out)
+    _check(_lib.psb_knn_bruteforce(index.handle, queries.data_ptr(), q, k, ids.data_ptr(),
+                                   dists.data_ptr(), _stream_handle(stream)), "psb_knn_bruteforce")
+    return ids, dists
+
+
+def psb_merge_topk(ids, dists, k: int, stream=None, out=None):
+    """ids/dists: CUDA [parts, q, k] -> (out_ids, out_dists) [q, k]."""
+    torch = _torch()
+    parts, q, kk = ids.shape
+    assert kk == k and dists.shape == ids.shape
+    ids, dists = ids.contiguous(), dists.contiguous()
+    if out is None:
+        out = (torch.empty((q, k), dtype=torch.int32, device=ids.device),
+               torch.empty((q, k), dtype=torch.float32, device=ids.device))
+    _check(_lib.psb_merge_topk(ids.data_ptr(), dists.data_ptr(), parts, q, k, out[0].data_ptr(),
+                               out[1].data_ptr(), _stream_handle(stream)), "psb_merge_topk")
+    return out
+
+
+def _parse_blob(buf: np.ndarray) -> dict:
+    hdr = buf[:64].view(np.int64)
+    n, d, F, L, H, id_base, total = (int(x) for x in hdr[:7])
+    o = 64
+    nlev = buf[o:o + 8 * (H + 1)].view(np.int64).copy()
+    o += 8 * (H + 1)
+    pts = buf[o:o + 4 * L * d * F].view(np.float32).reshape(L, d, F)
+    o += 4 * L * d * F
+    ids = buf[o:o + 4 * L * F].view(np.int32).reshape(L, F)
+    o += 4 * L * F
+    levels = {}
+    for lv in range(1, H + 1):
+        cnt = int(nlev[lv])
+        levels[lv] = buf[o:o + 4 * cnt * 2 * d * F].view(np.float32).reshape(cnt, d, 2, F)
+        o += 4 * cnt * 2 * d * F
+    return {"n": n, "d": d, "fanout": F, "leaves": L, "levels": H, "id_base": id_base,
+            "total_nodes": total, "nlev": nlev, "pts": pts, "ids": ids, "nodes": levels}
+
+
+def psb_index_export(index: Index) -> dict:
+    used = _i64()
+    _check(_lib.psb_index_export(index.handle, None, 0, ctypes.byref(used)), "psb_index_export")
+    buf = np.empty(used.value, dtype=np.uint8)
+    _check(_lib.psb_index_export(index.handle, buf.ctypes.data, used.value, ctypes.byref(used)),
+           "psb_index_export")
+    return _parse_blob(buf)
+
+
+def psb_build_host_blob(points, fanout: int, id_base: int = 0, packing: int = PSB_PACK_HILBERT,
+                        raw: bool = False):
+    """Host-only bulk load (no CUDA): the export blob of the index psb_build_ex would build."""
+    a = np.ascontiguousarray(points, dtype=np.float32)
+    used = _i64()
+    _check(_lib.psb_build_host_blob(a.ctypes.data, a.shape[0], a.shape[1], fanout, id_base, packing,
+                                    None, 0, ctypes.byref(used)), "psb_build_host_blob")
+    buf = np.empty(used.value, dtype=np.uint8)
+    _check(_lib.psb_build_host_blob(a.ctypes.data, a.shape[0], a.shape[1], fanout, id_base, packing,
+                                    buf.ctypes.data, used.value, ctypes.byref(used)), "psb_build_host_blob")
+    return buf if raw else _parse_blob(buf)
+
+
+def psb_free(index: Index):
+    index.free()
+
+
+def symbols_exported() -> dict:
+    """{symbol: bool} for every declared entry point (no compute calls)."""
+    out = {}
+    for s in EXPORTS:
+        try:
+            getattr(_lib, s)
+            out[s] = True
+        except AttributeError:
+            out[s] = False
+    return out

@@ -1,0 +1,315 @@
+// knn_tree.cu — the two tree traversals on sm_100a, one warp per query:
+//   psb_kernel : Parallel Scan and Backtrack (Alg. 1, §III)
+//   bnb_kernel : classic branch-and-bound (Roussopoulos [17]) made
+//                stackless with parent links as the paper ran it
+// Step names S1..S11 follow SURVEY.md §8(a); readings R1..R16 follow DESIGN.md §2.
+#include <cuda_runtime.h>
+
+#include "psb_device.cuh"
+#include "psb_launch.h"
+
+namespace psb {
+
+constexpr int WARPS_PER_CTA = 4;
+
+struct WarpState {
+    float *cache_md;     // [(H+1)][F] child MINDISTs of the node cached per level
+    int64_t *cache_node; // [(H+1)] node id cached per level (-1 = none)
+    float *qsmem;        // query (D == 0 only)
+};
+
+__device__ __forceinline__ WarpState warp_state(unsigned char *smem, int H, int F, bool qsmem)
+{
+    const int w = threadIdx.x >> 5;
+    unsigned char *base = smem + (size_t)w * WarpSmem::bytes(H, F, qsmem);
+    WarpState s;
+    s.cache_md = reinterpret_cast<float *>(base);
+    size_t off = (WarpSmem::cache_floats(H, F) * 4 + 15) & ~(size_t)15;
+    s.cache_node = reinterpret_cast<int64_t *>(base + off);
+    off += (size_t)(H + 1) * 8;
+    off = (off + 15) & ~(size_t)15;
+    s.qsmem = reinterpret_cast<float *>(base + off);
+    return s;
+}
+
+// S3+S4+S5 with the S7 path cache: child MINDISTs of internal node (lvl, node).
+// A node already cached at its level is not fetched again: MINDIST is a pure
+// function of (query, node), and its k-th-MAXDIST bound was applied when it was
+// first fetched (re-applying it could not lower pd further).
+template <int D, int V>
+__device__ __forceinline__ void internal_md(const DevIndex &ix, int lvl, int64_t node,
+                                            const Query<D> &q, int lane, const WarpState &ws,
+                                            bool use_cache, bool use_max, int k, float &pd,
+                                            float (&md)[V])
+{
+    constexpr int F = 32 * V;
+    float *cm = ws.cache_md + (size_t)lvl * F + lane * V;
+    if (use_cache && ws.cache_node[lvl] == node) {
+#pragma unroll
+        for (int t = 0; t < V; ++t) md[t] = cm[t];
+        return;
+    }
+    const float *blk = ix.nodes + ix.level_off[lvl] + node * ((int64_t)2 * ix.d * F);
+    float Md[V];
+    if (use_max) {
+        node_bounds<D, V, true>(blk, q, ix.d, lane, md, Md);
+        pd = kth_bound<V>(Md, k, pd);                    // Alg. 1 l.13-15
+    } else {
+        node_bounds<D, V, false>(blk, q, ix.d, lane, md, Md);
+    }
+    if (use_cache) {
+#pragma unroll
+        for (int t = 0; t < V; ++t) cm[t] = md[t];
+        __syncwarp();
+        if (lane == 0) ws.cache_node[lvl] = node;
+        __syncwarp();
+    }
+}
+
+__device__ __forceinline__ int64_t max_leaf(const DevIndex &ix, int lvl, int64_t node)
+{
+    const int64_t e = (node + 1) * ix.span[lvl];
+    return (e < ix.L ? e : ix.L) - 1;
+}
+
+template <int D, int V, int KS>
+__global__ void __launch_bounds__(WARPS_PER_CTA * 32)
+psb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
+           int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant)
+{
+    constexpr int F = 32 * V;
+    extern __shared__ __align__(16) unsigned char smem[];
+    const int lane = threadIdx.x & 31;
+    const int64_t qi = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
+    if (qi >= nq) return;
+    const int H = ix.H;
+    const WarpState ws = warp_state(smem, H, F, D == 0);
+    const bool use_cache = !(variant & PSB_VAR_NOCACHE);
+    const bool use_max = !(variant & PSB_VAR_NOMAXDIST);
+
+    // S1: query to registers, kNNs <- {inf} (Alg. 1 l.1-2)
+    Query<D> q;
+    q.load(queries + qi * ix.d, ix.d, ws.qsmem);
+    for (int l = lane; l <= H; l += 32) ws.cache_node[l] = -1;
+    __syncwarp();
+    TopK<KS> T;
+    T.init();
+    u64 thr = PAD_KEY;
+    float pd = __int_as_float(0x7f800000);
+
+    // S2: pass 1, getInitialPruningDistance(Q, ClosestLeaf) (Alg. 1 l.3; R4):
+    // greedy descent by (MINDIST, child index) argmin, k-th-MAXDIST bounds on the way.
+    int lvl = H;
+    int64_t node = 0;
+    while (lvl > 0) {
+        float md[V];
+        internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
+        const int64_t base = node * F, nb = ix.nlev[lvl - 1];
+        u64 best = ~0ull;
+#pragma unroll
+        for (int t = 0; t < V; ++t) {
+            const int c = lane * V + t;
+            if (base + c < nb) {
+                const u64 kk = make_key(md[t], c);
+                best = kk < best ? kk : best;
+            }
+        }
+        best = warp_min_u64(best);
+        node = base + (int64_t)(best & 0xffffffffu);
+        --lvl;
+    }
+    // ClosestLeaf and its right siblings until k points are seen; their points go
+    // straight into the kNN list (allowed by R4: pass 2 then skips these leaves).
+    const int64_t pass1_lo = node;
+    int64_t pass1_hi = node - 1, seen = 0;
+    while (seen < k && pass1_hi + 1 < ix.L) {
+        ++pass1_hi;
+        scan_leaf<D, V, KS>(ix, pass1_hi, q, lane, T, k, thr);
+        const int64_t left = ix.n - pass1_hi * F;
+        seen += left < F ? left : F;
+    }
+    pd = fminf(pd, key_dist(thr));
+
+    // Pass 2 (Alg. 1 l.6-47): leftmost eligible descent, left-to-right leaf scan,
+    // parent-link backtrack.
+    lvl = H;
+    node = 0;
+    int64_t visited = -1;                                        // R10
+    while (true) {
+        if (lvl > 0) {
+            float md[V];
+            internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
+            // S6: eligible(c) = MINDIST <= pd (R5) and unvisited leaves below (R8)
+            const int64_t base = node * F, nb = ix.nlev[lvl - 1];
+            unsigned mine = 0;
+#pragma unroll
+            for (int t = 0; t < V; ++t) {
+                const int64_t g = base + lane * V + t;
+                const bool e = g < nb && md[t] <= pd && max_leaf(ix, lvl - 1, g) > visited;
+                mine |= (unsigned)e << t;
+            }
+            const unsigned bal = __ballot_sync(FULL, mine != 0);
+            if (bal) {                                           // leftmost (R6, R7)
+                const int src = __ffs(bal) - 1;
+                const unsigned m = __shfl_sync(FULL, mine, src);
+                node = base + src * V + (__ffs(m) - 1);
+                --lvl;
+            } else {                                             // S7 backtrack (R9)
+                visited = max_leaf(ix, lvl, node);
+                if (lvl == H) break;
+                node /= F;
+                ++lvl;
+            }
+        } else {
+            // S8-S10: leaf j
+            const int64_t j = node;
+            bool changed;
+            if (j >= pass1_lo && j <= pass1_hi) {
+                changed = true;                                  // already offered in pass 1
+            } else {
+                changed = scan_leaf<D, V, KS>(ix, j, q, lane, T, k, thr);
+            }
+            pd = fminf(pd, key_dist(thr));                       // Alg. 1 l.37
+            visited = j;                                         // l.38
+            if (j == ix.L - 1) break;                            // R10
+            if (changed) {
+                node = j + 1;                                    // l.41 right sibling (R11, R12)
+            } else {
+                node = j / F;                                    // l.44 parent link
+                lvl = 1;
+            }
+        }
+    }
+    // S11
+    T.store(k, lane, out_ids + qi * k, out_dists + qi * k);
+}
+
+// Stackless B&B: at an internal node take the next child in
+// (MINDIST, index) order after the one we returned from, among those with
+// MINDIST <= pd; a leaf always returns to its parent.
+template <int D, int V, int KS>
+__global__ void __launch_bounds__(WARPS_PER_CTA * 32)
+bnb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
+           int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant)
+{
+    constexpr int F = 32 * V;
+    extern __shared__ __align__(16) unsigned char smem[];
+    const int lane = threadIdx.x & 31;
+    const int64_t qi = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
+    if (qi >= nq) return;
+    const int H = ix.H;
+    const WarpState ws = warp_state(smem, H, F, D == 0);
+    const bool use_cache = !(variant & PSB_VAR_NOCACHE);
+    const bool use_max = !(variant & PSB_VAR_NOMAXDIST);
+
+    Query<D> q;
+    q.load(queries + qi * ix.d, ix.d, ws.qsmem);
+    for (int l = lane; l <= H; l += 32) ws.cache_node[l] = -1;
+    __syncwarp();
+    TopK<KS> T;
+    T.init();
+    u64 thr = PAD_KEY;
+    float pd = __int_as_float(0x7f800000);
+
+    int lvl = H;
+    int64_t node = 0;
+    int from_c = -1;                        // child we returned from, -1 = fresh visit
+    while (true) {
+        if (lvl > 0) {
+            float md[V];
+            internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
+            u64 from_key = 0;
+            if (from_c >= 0) {
+                float v = md[0];
+#pragma unroll
+                for (int t = 1; t < V; ++t)
+                    if (t == from_c % V) v = md[t];
+                from_key = make_key(__shfl_sync(FULL, v, from_c / V), from_c);
+            }
+            const int64_t base = node * F, nb = ix.nlev[lvl - 1];
+            u64 best = ~0ull;
+#pragma unroll
+            for (int t = 0; t < V; ++t) {
+                const int c = lane * V + t;
+                const u64 kk = make_key(md[t], c);
+                if (base + c < nb && md[t] <= pd && (from_c < 0 || kk > from_key))
+                    best = kk < best ? kk : best;
+            }
+            best = warp_min_u64(best);
+            if (best != ~0ull) {
+                node = base + (int64_t)(best & 0xffffffffu);
+                --lvl;
+                from_c = -1;
+            } else {
+                if (lvl == H) break;
+                from_c = (int)(node % F);
+                node /= F;
+                ++lvl;
+            }
+        } else {
+            scan_leaf<D, V, KS>(ix, node, q, lane, T, k, thr);
+            pd = fminf(pd, key_dist(thr));
+            from_c = (int)(node % F);
+            node /= F;
+            lvl = 1;
+        }
+    }
+    T.store(k, lane, out_ids + qi * k, out_dists + qi * k);
+}
+
+template <int D, int V, int KS>
+static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
+                         int32_t *oi, float *od, cudaStream_t st, uint32_t variant)
+{
+    const size_t smem = WARPS_PER_CTA * WarpSmem::bytes(ix.H, 32 * V, D == 0);
+    const int64_t blocks = (nq + WARPS_PER_CTA - 1) / WARPS_PER_CTA;
+    auto kern = algo == PSB_ALGO_PSB ? psb_kernel<D, V, KS> : bnb_kernel<D, V, KS>;
+    if (smem > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return report_cuda(e, "cudaFuncSetAttribute");
+    }
+    kern<<<(unsigned)blocks, WARPS_PER_CTA * 32, smem, st>>>(ix, queries, nq, k, oi, od, variant);
+    return report_cuda(cudaGetLastError(), "tree kernel launch");
+}
+
+template <int D, int V>
+static int launch_tree_ks(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
+                          int32_t *oi, float *od, cudaStream_t st, uint32_t variant)
+{
+    if (k <= 32) return launch_tree_t<D, V, 1>(algo, ix, queries, nq, k, oi, od, st, variant);
+    if (k <= 64) return launch_tree_t<D, V, 2>(algo, ix, queries, nq, k, oi, od, st, variant);
+    return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant);
+}
+
+template <int D>
+static int launch_tree_v(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
+                         int32_t *oi, float *od, cudaStream_t st, uint32_t variant)
+{
+    switch (ix.F) {
+    case 32: return launch_tree_ks<D, 1>(algo, ix, queries, nq, k, oi, od, st, variant);
+    case 64: return launch_tree_ks<D, 2>(algo, ix, queries, nq, k, oi, od, st, variant);
+    case 128: return launch_tree_ks<D, 4>(algo, ix, queries, nq, k, oi, od, st, variant);
+    default: break;
+    }
+    if constexpr (D == 0) {
+        if (ix.F == 256) return launch_tree_ks<0, 8>(algo, ix, queries, nq, k, oi, od, st, variant);
+        if (ix.F == 512) return launch_tree_ks<0, 16>(algo, ix, queries, nq, k, oi, od, st, variant);
+        return PSB_EUNSUPPORTED;
+    } else {
+        return launch_tree_v<0>(algo, ix, queries, nq, k, oi, od, st, variant);
+    }
+}
+
+int launch_tree(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
+                float *od, cudaStream_t st, uint32_t variant)
+{
+    switch (ix.d) {
+    case 2: return launch_tree_v<2>(algo, ix, queries, nq, k, oi, od, st, variant);
+    case 3: return launch_tree_v<3>(algo, ix, queries, nq, k, oi, od, st, variant);
+    case 8: return launch_tree_v<8>(algo, ix, queries, nq, k, oi, od, st, variant);
+    case 16: return launch_tree_v<16>(algo, ix, queries, nq, k, oi, od, st, variant);
+    default: return launch_tree_v<0>(algo, ix, queries, nq, k, oi, od, st, variant);
+    }
+}
+
+}  // namespace psb

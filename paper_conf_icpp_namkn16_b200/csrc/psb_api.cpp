@@ -1,0 +1,308 @@
+// psb_api.cpp — the C ABI of libpsb.so (declared and documented in include/psb.h):
+// argument validation, index upload, kernel dispatch, error reporting.
+#include <cuda_runtime.h>
+
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+
+#include "psb_internal.h"
+#include "psb_launch.h"
+
+#ifndef PSB_VERSION
+#define PSB_VERSION "0.1.0"
+#endif
+
+static thread_local char g_err[512];
+
+void psb_set_error(const char *fmt, ...)
+{
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof g_err, fmt, ap);
+    va_end(ap);
+}
+
+namespace psb {
+int report_cuda(cudaError_t e, const char *what)
+{
+    if (e == cudaSuccess) return PSB_OK;
+    psb_set_error("%s: %s (%s)", what, cudaGetErrorString(e), cudaGetErrorName(e));
+    return e == cudaErrorMemoryAllocation ? PSB_ENOMEM : PSB_ECUDA;
+}
+}  // namespace psb
+using psb::report_cuda;
+
+struct psb_index {
+    int device = -1;
+    int sm_count = 0;
+    int64_t n = 0, L = 0, id_base = 0;
+    int32_t d = 0, F = 0, H = 0;
+    int64_t nlev[PSB_MAXLVL + 1] = {};
+    int64_t level_off[PSB_MAXLVL + 1] = {};
+    int64_t node_floats = 0;
+    float *pts = nullptr;
+    int32_t *ids = nullptr;
+    float *nodes = nullptr;
+    int64_t device_bytes = 0;
+};
+
+static void index_release(psb_index *ix)
+{
+    if (!ix) return;
+    int prev = -1;
+    cudaGetDevice(&prev);
+    if (ix->device >= 0) cudaSetDevice(ix->device);
+    cudaFree(ix->pts);
+    cudaFree(ix->ids);
+    cudaFree(ix->nodes);
+    if (prev >= 0) cudaSetDevice(prev);
+    delete ix;
+}
+
+static DevIndex dev_view(const psb_index *ix)
+{
+    DevIndex v;
+    memset(&v, 0, sizeof v);
+    v.pts = ix->pts;
+    v.ids = ix->ids;
+    v.nodes = ix->nodes;
+    for (int l = 0; l <= PSB_MAXLVL; ++l) {
+        v.level_off[l] = ix->level_off[l];
+        v.nlev[l] = ix->nlev[l];
+    }
+    int64_t s = 1;
+    for (int l = 0; l <= PSB_MAXLVL; ++l) {
+        v.span[l] = s < ix->L ? s : ix->L;   // F^l clamped at L (only the root reaches it)
+        if (s < ix->L) s *= ix->F;
+    }
+    v.n = ix->n;
+    v.L = ix->L;
+    v.H = ix->H;
+    v.d = ix->d;
+    v.F = ix->F;
+    return v;
+}
+
+extern "C" {
+
+const char *psb_last_error(void) { return g_err; }
+
+const char *psb_version(void) { return "psb-b200 " PSB_VERSION " sm_100a"; }
+
+int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int64_t id_base,
+                 uint32_t flags, psb_index **out)
+{
+    g_err[0] = 0;
+    if (!out) { psb_set_error("psb_build_ex: out is NULL"); return PSB_EINVAL; }
+    *out = nullptr;
+    if (!points) { psb_set_error("psb_build_ex: points is NULL"); return PSB_EINVAL; }
+    if (n < 1 || d < 1 || d > PSB_DMAX) {
+        psb_set_error("psb_build_ex: n=%lld d=%d out of range", (long long)n, d);
+        return PSB_EINVAL;
+    }
+    int dev = -1;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return report_cuda(e, "psb_build_ex: cudaGetDevice");
+    // points may be host or device memory; the bulk load runs on the host
+    cudaPointerAttributes attr;
+    const float *host_pts = points;
+    float *staged = nullptr;
+    e = cudaPointerGetAttributes(&attr, points);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        attr.type = cudaMemoryTypeUnregistered;
+    }
+    if (attr.type == cudaMemoryTypeDevice) {
+        staged = (float *)malloc(sizeof(float) * (size_t)(n * d));
+        if (!staged) { psb_set_error("psb_build_ex: host staging allocation failed"); return PSB_ENOMEM; }
+        e = cudaMemcpy(staged, points, sizeof(float) * (size_t)(n * d), cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) { free(staged); return report_cuda(e, "psb_build_ex: copy points to host"); }
+        host_pts = staged;
+    }
+    HostLayout h;
+    int rc = psb_host_build(host_pts, n, d, fanout, id_base, flags, &h);
+    free(staged);
+    if (rc != PSB_OK) return rc;
+
+    psb_index *ix = new (std::nothrow) psb_index;
+    if (!ix) { psb_set_error("psb_build_ex: host allocation failed"); return PSB_ENOMEM; }
+    ix->device = dev;
+    cudaDeviceGetAttribute(&ix->sm_count, cudaDevAttrMultiProcessorCount, dev);
+    ix->n = h.n; ix->L = h.L; ix->id_base = h.id_base;
+    ix->d = h.d; ix->F = h.F; ix->H = h.H;
+    for (int l = 0; l <= PSB_MAXLVL; ++l) { ix->nlev[l] = h.nlev[l]; ix->level_off[l] = h.level_off[l]; }
+    ix->node_floats = h.total_node_floats;
+    const size_t bp = sizeof(float) * (size_t)(h.L * d * fanout);
+    const size_t bi = sizeof(int32_t) * (size_t)(h.L * fanout);
+    const size_t bn = sizeof(float) * (size_t)h.total_node_floats;
+    if ((e = cudaMalloc((void **)&ix->pts, bp)) != cudaSuccess ||
+        (e = cudaMalloc((void **)&ix->ids, bi)) != cudaSuccess ||
+        (e = cudaMalloc((void **)&ix->nodes, bn)) != cudaSuccess ||
+        (e = cudaMemcpy(ix->pts, h.pts, bp, cudaMemcpyHostToDevice)) != cudaSuccess ||
+        (e = cudaMemcpy(ix->ids, h.ids, bi, cudaMemcpyHostToDevice)) != cudaSuccess ||
+        (e = cudaMemcpy(ix->nodes, h.nodes, bn, cudaMemcpyHostToDevice)) != cudaSuccess) {
+        rc = report_cuda(e, "psb_build_ex: upload");
+        index_release(ix);
+        return rc;
+    }
+    ix->device_bytes = (int64_t)(bp + bi + bn);
+    *out = ix;
+    return PSB_OK;
+}
+
+psb_index *psb_build(const float *points, int64_t n, int32_t d, int32_t fanout)
+{
+    psb_index *ix = nullptr;
+    return psb_build_ex(points, n, d, fanout, 0, PSB_PACK_HILBERT, &ix) == PSB_OK ? ix : nullptr;
+}
+
+void psb_free(psb_index *ix) { index_release(ix); }
+
+static int check_query_args(const char *fn, const psb_index *ix, const float *queries, int64_t q,
+                            int32_t k, const void *oi, const void *od)
+{
+    if (!ix) { psb_set_error("%s: index is NULL", fn); return PSB_EINVAL; }
+    if (q < 0) { psb_set_error("%s: q=%lld < 0", fn, (long long)q); return PSB_EINVAL; }
+    if (k < 1) { psb_set_error("%s: k=%d < 1", fn, k); return PSB_EINVAL; }
+    if (k > PSB_KMAX) { psb_set_error("%s: k=%d > PSB_KMAX=%d", fn, k, PSB_KMAX); return PSB_EUNSUPPORTED; }
+    if (q > 0 && (!queries || !oi || !od)) { psb_set_error("%s: NULL buffer", fn); return PSB_EINVAL; }
+    if (q > ((int64_t)1 << 40)) { psb_set_error("%s: q=%lld too large", fn, (long long)q); return PSB_EINVAL; }
+    int dev = -1;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return report_cuda(e, fn);
+    if (dev != ix->device) {
+        psb_set_error("%s: index lives on device %d but device %d is current", fn, ix->device, dev);
+        return PSB_EINVAL;
+    }
+    return PSB_OK;
+}
+
+int psb_knn_ex(const psb_index *ix, const float *queries, int64_t q, int32_t k, int32_t *out_ids,
+               float *out_dists, void *stream, int32_t algo, uint32_t variant)
+{
+    g_err[0] = 0;
+    int rc = check_query_args("psb_knn", ix, queries, q, k, out_ids, out_dists);
+    if (rc != PSB_OK) return rc;
+    if (variant & ~(uint32_t)(PSB_VAR_NOCACHE | PSB_VAR_NOMAXDIST)) {
+        psb_set_error("psb_knn_ex: unknown variant bits 0x%x", variant);
+        return PSB_EINVAL;
+    }
+    if (q == 0) return PSB_OK;
+    const DevIndex v = dev_view(ix);
+    cudaStream_t st = (cudaStream_t)stream;
+    switch (algo) {
+    case PSB_ALGO_PSB:
+    case PSB_ALGO_BNB: return psb::launch_tree(algo, v, queries, q, k, out_ids, out_dists, st, variant);
+    case PSB_ALGO_BRUTE: return psb::launch_brute(v, queries, q, k, out_ids, out_dists, st, ix->sm_count);
+    default: psb_set_error("psb_knn_ex: unknown algo %d", algo); return PSB_EINVAL;
+    }
+}
+
+int psb_knn(const psb_index *ix, const float *queries, int64_t q, int32_t k, int32_t *out_ids,
+            float *out_dists, void *stream)
+{
+    return psb_knn_ex(ix, queries, q, k, out_ids, out_dists, stream, PSB_ALGO_PSB, 0);
+}
+
+int psb_knn_branch_and_bound(const psb_index *ix, const float *queries, int64_t q, int32_t k,
+                             int32_t *out_ids, float *out_dists, void *stream)
+{
+    return psb_knn_ex(ix, queries, q, k, out_ids, out_dists, stream, PSB_ALGO_BNB, 0);
+}
+
+int psb_knn_bruteforce(const psb_index *ix, const float *queries, int64_t q, int32_t k,
+                       int32_t *out_ids, float *out_dists, void *stream)
+{
+    return psb_knn_ex(ix, queries, q, k, out_ids, out_dists, stream, PSB_ALGO_BRUTE, 0);
+}
+
+int psb_merge_topk(const int32_t *ids, const float *dists, int32_t parts, int64_t q, int32_t k,
+                   int32_t *out_ids, float *out_dists, void *stream)
+{
+    g_err[0] = 0;
+    if (parts < 1 || q < 0 || k < 1) {
+        psb_set_error("psb_merge_topk: parts=%d q=%lld k=%d out of range", parts, (long long)q, k);
+        return PSB_EINVAL;
+    }
+    if (k > PSB_KMAX) { psb_set_error("psb_merge_topk: k=%d > PSB_KMAX", k); return PSB_EUNSUPPORTED; }
+    if (q == 0) return PSB_OK;
+    if (!ids || !dists || !out_ids || !out_dists) { psb_set_error("psb_merge_topk: NULL buffer"); return PSB_EINVAL; }
+    return psb::launch_merge(ids, dists, parts, q, k, out_ids, out_dists, (cudaStream_t)stream);
+}
+
+int psb_index_info(const psb_index *ix, int64_t *n, int32_t *d, int32_t *fanout, int64_t *leaves,
+                   int32_t *levels, int64_t *device_bytes)
+{
+    if (!ix) { psb_set_error("psb_index_info: index is NULL"); return PSB_EINVAL; }
+    if (n) *n = ix->n;
+    if (d) *d = ix->d;
+    if (fanout) *fanout = ix->F;
+    if (leaves) *leaves = ix->L;
+    if (levels) *levels = ix->H;
+    if (device_bytes) *device_bytes = ix->device_bytes;
+    return PSB_OK;
+}
+
+static int64_t blob_size(int64_t L, int32_t d, int32_t F, int32_t H, int64_t node_floats)
+{
+    return 8 * 8 + 8 * (int64_t)(H + 1) + 4 * L * d * F + 4 * L * F + 4 * node_floats;
+}
+
+static void blob_header(char *buf, int64_t n, int32_t d, int32_t F, int64_t L, int32_t H, int64_t id_base,
+                        const int64_t *nlev)
+{
+    int64_t total = 0;
+    for (int l = 1; l <= H; ++l) total += nlev[l];
+    int64_t hdr[8] = {n, d, F, L, H, id_base, total, 0};
+    memcpy(buf, hdr, sizeof hdr);
+    memcpy(buf + sizeof hdr, nlev, 8 * (size_t)(H + 1));
+}
+
+int psb_index_export(const psb_index *ix, void *host_buf, int64_t cap, int64_t *used)
+{
+    if (!ix || !used) { psb_set_error("psb_index_export: NULL argument"); return PSB_EINVAL; }
+    const int64_t need = blob_size(ix->L, ix->d, ix->F, ix->H, ix->node_floats);
+    *used = need;
+    if (!host_buf) return PSB_OK;
+    if (cap < need) { psb_set_error("psb_index_export: cap %lld < %lld", (long long)cap, (long long)need); return PSB_EINVAL; }
+    char *b = (char *)host_buf;
+    blob_header(b, ix->n, ix->d, ix->F, ix->L, ix->H, ix->id_base, ix->nlev);
+    char *p = b + 64 + 8 * (ix->H + 1);
+    const size_t bp = 4 * (size_t)(ix->L * ix->d * ix->F), bi = 4 * (size_t)(ix->L * ix->F);
+    cudaError_t e;
+    if ((e = cudaMemcpy(p, ix->pts, bp, cudaMemcpyDeviceToHost)) != cudaSuccess ||
+        (e = cudaMemcpy(p + bp, ix->ids, bi, cudaMemcpyDeviceToHost)) != cudaSuccess ||
+        (e = cudaMemcpy(p + bp + bi, ix->nodes, 4 * (size_t)ix->node_floats, cudaMemcpyDeviceToHost)) != cudaSuccess)
+        return report_cuda(e, "psb_index_export");
+    return PSB_OK;
+}
+
+// Host-only bulk load into the export blob layout (no CUDA calls): lets the CPU
+// test suite check the layout logic; the GPU tests check psb_index_export of a
+// real index against it.
+int psb_build_host_blob(const float *points, int64_t n, int32_t d, int32_t fanout, int64_t id_base,
+                        uint32_t flags, void *host_buf, int64_t cap, int64_t *used)
+{
+    g_err[0] = 0;
+    if (!used) { psb_set_error("psb_build_host_blob: used is NULL"); return PSB_EINVAL; }
+    HostLayout h;
+    int rc = psb_host_build(points, n, d, fanout, id_base, flags, &h);
+    if (rc != PSB_OK) return rc;
+    const int64_t need = blob_size(h.L, h.d, h.F, h.H, h.total_node_floats);
+    *used = need;
+    if (!host_buf) return PSB_OK;
+    if (cap < need) { psb_set_error("psb_build_host_blob: cap too small"); return PSB_EINVAL; }
+    char *b = (char *)host_buf;
+    blob_header(b, h.n, h.d, h.F, h.L, h.H, h.id_base, h.nlev);
+    char *p = b + 64 + 8 * (h.H + 1);
+    const size_t bp = 4 * (size_t)(h.L * h.d * h.F), bi = 4 * (size_t)(h.L * h.F);
+    memcpy(p, h.pts, bp);
+    memcpy(p + bp, h.ids, bi);
+    memcpy(p + bp + bi, h.nodes, 4 * (size_t)h.total_node_floats);
+    return PSB_OK;
+}
+
+}  // extern "C"

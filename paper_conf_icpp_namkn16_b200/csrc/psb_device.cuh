@@ -1,0 +1,292 @@
+// psb_device.cuh — warp-level building blocks of the sm_100a kNN kernels.
+//
+// One warp owns one query. For a node (or leaf) of fanout F = 32*V, lane l owns
+// the V consecutive children (points) l*V .. l*V+V-1, so each SoA row of F
+// floats is read by the warp as one fully coalesced 128-bit (V=4), 64-bit (V=2)
+// or 32-bit (V=1) load per lane ("SoA so that memory coalescing can be naturally
+// employed", §V-A; "parfor tid <- 1, numChildNodes",
+// Alg. 1 l.9-12).
+//
+// Arithmetic is binary32 with every operation explicitly rounded to nearest
+// (__fsub_rn/__fmul_rn/__fadd_rn: never contracted to FMA, never flushed to
+// zero), dimensions in order — the distance the oracle defines.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "psb_internal.h"
+
+namespace psb {
+
+typedef unsigned long long u64;
+constexpr unsigned FULL = 0xffffffffu;
+// (dist, id) packed as one u64 key: for dist >= +0 the IEEE bit pattern orders
+// like the value, so u64 order == lexicographic (dist, id) order for ids >= 0.
+// The pad (+inf, -1) = 0x7F800000FFFFFFFF is larger than every real key.
+constexpr u64 PAD_KEY = 0x7F800000FFFFFFFFull;
+
+__device__ __forceinline__ u64 make_key(float d, int32_t id)
+{
+    return ((u64)__float_as_uint(d) << 32) | (u64)(uint32_t)id;
+}
+__device__ __forceinline__ float key_dist(u64 k) { return __uint_as_float((uint32_t)(k >> 32)); }
+__device__ __forceinline__ int32_t key_id(u64 k) { return (int32_t)(uint32_t)(k & 0xffffffffu); }
+
+// (a - b)^2, each op rounded once.
+__device__ __forceinline__ float sq_diff(float a, float b)
+{
+    float t = __fsub_rn(a, b);
+    return __fmul_rn(t, t);
+}
+
+// Loop over dimensions 0..d-1 in order: fully unrolled for a compile-time D (so
+// query coordinates stay in registers), a runtime loop otherwise.
+template <int D, typename Body>
+__device__ __forceinline__ void for_dims(int d, Body &&body)
+{
+    if constexpr (D > 0) {
+#pragma unroll
+        for (int j = 0; j < D; ++j) body(j);
+    } else {
+#pragma unroll 2
+        for (int j = 0; j < d; ++j) body(j);
+    }
+}
+
+// V consecutive floats, V*4-byte aligned, read-only path.
+template <int V>
+__device__ __forceinline__ void ldv(const float *__restrict__ p, float (&o)[V])
+{
+    if constexpr (V == 1) {
+        o[0] = __ldg(p);
+    } else if constexpr (V == 2) {
+        float2 x = __ldg(reinterpret_cast<const float2 *>(p));
+        o[0] = x.x; o[1] = x.y;
+    } else {
+#pragma unroll
+        for (int i = 0; i < V; i += 4) {
+            float4 x = __ldg(reinterpret_cast<const float4 *>(p + i));
+            o[i] = x.x; o[i + 1] = x.y; o[i + 2] = x.z; o[i + 3] = x.w;
+        }
+    }
+}
+
+// Query coordinates: registers for a compile-time D, shared memory otherwise.
+template <int D>
+struct Query {
+    float c[D];
+    __device__ __forceinline__ void load(const float *__restrict__ q, int, float *)
+    {
+#pragma unroll
+        for (int j = 0; j < D; ++j) c[j] = __ldg(q + j);
+    }
+    __device__ __forceinline__ float operator[](int j) const { return c[j]; }
+};
+template <>
+struct Query<0> {
+    const float *s;
+    __device__ __forceinline__ void load(const float *__restrict__ q, int d, float *smem)
+    {
+        for (int j = threadIdx.x & 31; j < d; j += 32) smem[j] = __ldg(q + j);
+        __syncwarp();
+        s = smem;
+    }
+    __device__ __forceinline__ float operator[](int j) const { return s[j]; }
+};
+
+// S4: MINDIST and MAXDIST of the query to this lane's V child
+// MBRs of one node block [d][2][F] (Alg. 1 l.9-12, §III).
+//   MINDIST term: lo-q if q<lo, q-hi if q>hi, else 0;  MAXDIST term: max(|q-lo|,|q-hi|)
+// Empty slots (lo=+inf, hi=-inf) give +inf for both.
+template <int D, int V, bool MAX>
+__device__ __forceinline__ void node_bounds(const float *__restrict__ blk, const Query<D> &q, int d,
+                                            int lane, float (&md)[V], float (&Md)[V])
+{
+    constexpr int F = 32 * V;
+#pragma unroll
+    for (int t = 0; t < V; ++t) { md[t] = 0.f; Md[t] = 0.f; }
+    for_dims<D>(d, [&](int j) {
+        float lo[V], hi[V];
+        ldv<V>(blk + (2 * j) * F + lane * V, lo);
+        ldv<V>(blk + (2 * j + 1) * F + lane * V, hi);
+        const float qj = q[j];
+#pragma unroll
+        for (int t = 0; t < V; ++t) {
+            float a = __fsub_rn(lo[t], qj);   // lo - q   (= -(q - lo) exactly)
+            float b = __fsub_rn(qj, hi[t]);   // q - hi
+            float tm = qj < lo[t] ? a : (qj > hi[t] ? b : 0.f);
+            md[t] = __fadd_rn(md[t], __fmul_rn(tm, tm));
+            if (MAX) {
+                float tx = fmaxf(fabsf(a), fabsf(b));
+                Md[t] = __fadd_rn(Md[t], __fmul_rn(tx, tx));
+            }
+        }
+    });
+}
+
+// S8: distances of the query to this lane's V points of one leaf block [d][F].
+template <int D, int V>
+__device__ __forceinline__ void leaf_dists(const float *__restrict__ lp, const Query<D> &q, int d,
+                                           int lane, float (&dist)[V])
+{
+    constexpr int F = 32 * V;
+#pragma unroll
+    for (int t = 0; t < V; ++t) dist[t] = 0.f;
+    for_dims<D>(d, [&](int j) {
+        float p[V];
+        ldv<V>(lp + j * F + lane * V, p);
+        const float qj = q[j];
+#pragma unroll
+        for (int t = 0; t < V; ++t) dist[t] = __fadd_rn(dist[t], sq_diff(p[t], qj));
+    });
+}
+
+__device__ __forceinline__ u64 warp_min_u64(u64 v)
+{
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        u64 w = __shfl_xor_sync(FULL, v, o);
+        v = w < v ? w : v;
+    }
+    return v;
+}
+
+// S5: k-th smallest of the warp's F MAXDIST values if it is below `pd`, else pd
+// (Alg. 1 l.13-15 parReduceFindKthMinMaxDist). The k-th smallest
+// MAXDIST over k non-empty disjoint children bounds the k-th NN distance.
+// Cheap filter first: fewer than k values below pd cannot lower pd. Otherwise a
+// 31-step radix select on the (non-negative) float bit patterns.
+template <int V>
+__device__ __forceinline__ float kth_bound(const float (&Md)[V], int k, float pd)
+{
+    int c = 0;
+#pragma unroll
+    for (int t = 0; t < V; ++t) c += Md[t] < pd;
+    c = __reduce_add_sync(FULL, c);
+    if (c < k) return pd;
+    uint32_t res = 0;
+    for (int bit = 30; bit >= 0; --bit) {
+        const uint32_t trial = res | (1u << bit);
+        int n = 0;
+#pragma unroll
+        for (int t = 0; t < V; ++t) n += __float_as_uint(Md[t]) < trial;
+        n = __reduce_add_sync(FULL, n);
+        if (n < k) res = trial;
+    }
+    return __uint_as_float(res);
+}
+
+// Warp-distributed sorted top-k of u64 keys (S9; the paper keeps "the kNN list
+// and k pruning distances" in shared memory; here they live in
+// registers): position r = s*32 + lane holds the r-th smallest key, KS keys per
+// lane, k <= 32*KS. Positions >= k are scratch.
+template <int KS>
+struct TopK {
+    u64 key[KS];
+
+    __device__ __forceinline__ void init()
+    {
+#pragma unroll
+        for (int s = 0; s < KS; ++s) key[s] = PAD_KEY;
+    }
+    // key at position k-1 (the current k-th neighbour), warp-uniform
+    __device__ __forceinline__ u64 kth(int k) const
+    {
+        const int s = (k - 1) >> 5;
+        u64 v = key[0];
+#pragma unroll
+        for (int i = 1; i < KS; ++i)
+            if (i == s) v = key[i];
+        return __shfl_sync(FULL, v, (k - 1) & 31);
+    }
+    // insert warp-uniform x (x not already present); everything above shifts up
+    __device__ __forceinline__ void insert(u64 x, int lane)
+    {
+        int p = 0;
+#pragma unroll
+        for (int s = 0; s < KS; ++s) p += __popc(__ballot_sync(FULL, key[s] < x));
+        u64 prev[KS];
+#pragma unroll
+        for (int s = 0; s < KS; ++s) {
+            u64 up = __shfl_up_sync(FULL, key[s], 1);
+            u64 wrap = s ? __shfl_sync(FULL, key[s > 0 ? s - 1 : 0], 31) : x;
+            prev[s] = lane ? up : wrap;
+        }
+#pragma unroll
+        for (int s = 0; s < KS; ++s) {
+            const int r = s * 32 + lane;
+            key[s] = r > p ? prev[s] : (r == p ? x : key[s]);
+        }
+    }
+    // Offer this lane's V candidate keys (~0 = none); returns whether any entered
+    // the first k positions. `thr` is the k-th key, kept current.
+    template <int V>
+    __device__ __forceinline__ bool offer(const u64 (&cand)[V], int k, int lane, u64 &thr)
+    {
+        bool changed = false;
+#pragma unroll
+        for (int t = 0; t < V; ++t) {
+            unsigned m = __ballot_sync(FULL, cand[t] < thr);
+            while (m) {
+                const int src = __ffs(m) - 1;
+                m &= m - 1;
+                const u64 x = __shfl_sync(FULL, cand[t], src);
+                if (x < thr) {
+                    insert(x, lane);
+                    thr = kth(k);
+                    changed = true;
+                }
+            }
+        }
+        return changed;
+    }
+    __device__ __forceinline__ void store(int k, int lane, int32_t *__restrict__ oi,
+                                          float *__restrict__ od) const
+    {
+#pragma unroll
+        for (int s = 0; s < KS; ++s) {
+            const int r = s * 32 + lane;
+            if (r < k) {
+                oi[r] = key_id(key[s]);
+                od[r] = key_dist(key[s]);
+            }
+        }
+    }
+};
+
+// S8+S9: scan one leaf, offer its points. Ids are fetched lazily, only for
+// points whose distance can enter the list (dist <= current k-th distance).
+template <int D, int V, int KS>
+__device__ __forceinline__ bool scan_leaf(const DevIndex &ix, int64_t leaf, const Query<D> &q,
+                                          int lane, TopK<KS> &T, int k, u64 &thr)
+{
+    constexpr int F = 32 * V;
+    float dist[V];
+    leaf_dists<D, V>(ix.pts + leaf * (int64_t)ix.d * F, q, ix.d, lane, dist);
+    const float td = key_dist(thr);
+    bool any = false;
+#pragma unroll
+    for (int t = 0; t < V; ++t) any |= dist[t] <= td;
+    if (!__any_sync(FULL, any)) return false;
+    const int32_t *__restrict__ lid = ix.ids + leaf * F + lane * V;
+    u64 cand[V];
+#pragma unroll
+    for (int t = 0; t < V; ++t) cand[t] = dist[t] <= td ? make_key(dist[t], __ldg(lid + t)) : ~0ull;
+    return T.template offer<V>(cand, k, lane, thr);
+}
+
+// Per-warp shared-memory layout for the traversal kernels.
+struct WarpSmem {
+    static __host__ __device__ __forceinline__ size_t cache_floats(int H, int F) { return (size_t)(H + 1) * F; }
+    static __host__ __device__ __forceinline__ size_t bytes(int H, int F, bool qsmem)
+    {
+        size_t b = cache_floats(H, F) * 4;
+        b = (b + 15) & ~(size_t)15;
+        b += (size_t)(H + 1) * 8;
+        b = (b + 15) & ~(size_t)15;
+        if (qsmem) b += PSB_DMAX * 4;
+        return b;
+    }
+};
+
+}  // namespace psb

@@ -1,0 +1,26 @@
+// psb_launch.h — host-side launchers implemented in the .cu files.
+#pragma once
+#include <cuda_runtime.h>
+
+#include "psb_internal.h"
+
+namespace psb {
+
+// Records a CUDA error in psb_last_error and maps it to PSB_ECUDA.
+int report_cuda(cudaError_t e, const char *what);
+
+// PSB_ALGO_PSB or PSB_ALGO_BNB, one warp per query (knn_tree.cu).
+int launch_tree(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
+                float *od, cudaStream_t st, uint32_t variant);
+
+// Exhaustive scan of all points (knn_brute.cu). Splits the point set into
+// chunks when there are too few queries to fill the GPU and merges the partial
+// lists with launch_merge; scratch is stream-ordered.
+int launch_brute(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi, float *od,
+                 cudaStream_t st, int sm_count);
+
+// [parts][nq][k] sorted (dist, id) lists -> first k of their union (knn_brute.cu).
+int launch_merge(const int32_t *ids, const float *dists, int parts, int64_t nq, int k, int32_t *oi,
+                 float *od, cudaStream_t st);
+
+}  // namespace psb

@@ -1,0 +1,270 @@
+"""GPU parity: libpsb.so (through its C ABI via the thin binding) vs the CPU oracle.
+
+Bar (north_star): bit-exact ids AND bit-exact binary32 squared
+distances for every query compared. Small configs compare every query; the
+full BASELINE.json sizes compare every query against the oracle's B&B (itself
+pinned to the oracle's brute force) or a stated sample against brute force.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+ALGOS = ("psb", "bnb", "brute")
+
+
+def _psb():
+    import paper_conf_icpp_namkn16_b200 as psb
+    return psb
+
+
+def run(idx, qs, k, algo="psb", variant=0):
+    psb = _psb()
+    a = {"psb": psb.PSB_ALGO_PSB, "bnb": psb.PSB_ALGO_BNB, "brute": psb.PSB_ALGO_BRUTE}[algo]
+    qd = torch.from_numpy(np.ascontiguousarray(qs, np.float32)).cuda()
+    ids, d = psb.psb_knn_ex(idx, qd, k, algo=a, variant=variant)
+    torch.cuda.synchronize()
+    return ids.cpu().numpy(), d.cpu().numpy()
+
+
+def assert_same(got, exp, what=""):
+    gi, gd = got
+    ei, ed = exp
+    bad = np.nonzero((gi != ei).any(1) | (gd.view(np.uint32) != ed.view(np.uint32)).any(1))[0]
+    if len(bad):
+        r = bad[0]
+        raise AssertionError(f"{what}: {len(bad)} rows differ; first row {r}:\n gpu ids {gi[r][:12]}\n"
+                             f" exp ids {ei[r][:12]}\n gpu d {gd[r][:6]}\n exp d {ed[r][:6]}")
+
+
+@pytest.fixture(scope="module")
+def c1():
+    cfg = W.config("C1")
+    pts, qs = cfg.points(), cfg.queries()
+    idx = _psb().psb_build(pts, cfg.fanout)
+    exp = oracle.knn_bruteforce(pts, qs, cfg.k)
+    yield cfg, pts, qs, idx, exp
+    idx.free()
+
+
+@pytest.mark.parametrize("algo", ALGOS)
+def test_c1_all_queries(c1, algo):
+    cfg, pts, qs, idx, exp = c1
+    assert_same(run(idx, qs, cfg.k, algo), exp, f"C1 {algo}")
+
+
+@pytest.mark.parametrize("variant", [1, 2, 3])
+@pytest.mark.parametrize("algo", ["psb", "bnb"])
+def test_c1_variants(c1, algo, variant):
+    cfg, pts, qs, idx, exp = c1
+    assert_same(run(idx, qs, cfg.k, algo, variant), exp, f"C1 {algo} var{variant}")
+
+
+@pytest.mark.parametrize("k", [1, 2, 31, 32, 33, 64, 65, 100, 128])
+def test_c1_k_sweep(c1, k):
+    cfg, pts, qs, idx, _ = c1
+    exp = oracle.knn_bruteforce(pts, qs, k)
+    for algo in ALGOS:
+        assert_same(run(idx, qs, k, algo), exp, f"C1 k={k} {algo}")
+
+
+@pytest.fixture(scope="module")
+def c2():
+    cfg = W.config("C2")
+    pts, qs = cfg.points(), cfg.queries()
+    idx = _psb().psb_build(pts, cfg.fanout)
+    tree = oracle.Tree(pts)
+    exp = tree.knn(qs, cfg.k)
+    yield cfg, pts, qs, idx, exp
+    idx.free()
+
+
+def test_c2_oracle_routes_agree_on_sample(c2):
+    cfg, pts, qs, idx, exp = c2
+    s = np.arange(0, cfg.q, 97)
+    bf = oracle.knn_bruteforce(pts, qs[s], cfg.k)
+    assert_same(bf, (exp[0][s], exp[1][s]), "oracle brute vs oracle bnb")
+
+
+@pytest.mark.parametrize("algo", ALGOS)
+def test_c2_full_all_queries(c2, algo):
+    """BASELINE.json configs[1]: 3-D clustered n=1M F=64 q=10^4 k=32, every query,
+    in the launch configuration bench.py times."""
+    cfg, pts, qs, idx, exp = c2
+    assert_same(run(idx, qs, cfg.k, algo), exp, f"C2 {algo}")
+
+
+def test_c2_nocache_and_batches(c2):
+    cfg, pts, qs, idx, exp = c2
+    sl = slice(0, 3000)
+    assert_same(run(idx, qs[sl], cfg.k, "psb", 1), (exp[0][sl], exp[1][sl]), "C2 psb nocache")
+    # batching/order independence: single queries and a reversed batch
+    for i in (0, 17, 4999):
+        assert_same(run(idx, qs[i:i + 1], cfg.k), (exp[0][i:i + 1], exp[1][i:i + 1]), "C2 single")
+    r = run(idx, qs[::-1][:2000], cfg.k)
+    assert_same(r, (exp[0][::-1][:2000], exp[1][::-1][:2000]), "C2 reversed")
+
+
+def test_c3_sampled():
+    """configs[2]: 8-D uniform n=4M F=128 k=16; a 2,000-query sample of the 10^5."""
+    cfg = W.config("C3")
+    pts = cfg.points()
+    qs = cfg.queries(q=2000)
+    idx = _psb().psb_build(pts, cfg.fanout)
+    exp = oracle.Tree(pts).knn(qs, cfg.k)
+    for algo in ALGOS:
+        assert_same(run(idx, qs, cfg.k, algo), exp, f"C3 {algo}")
+    bf = oracle.knn_bruteforce(pts, qs[:40], cfg.k)
+    assert_same(run(idx, qs[:40], cfg.k), bf, "C3 psb vs oracle brute")
+    idx.free()
+
+
+def test_c4_sampled():
+    """configs[3]: 16-D clustered n=16M F=128 k=64; 200 sampled queries."""
+    cfg = W.config("C4")
+    pts = cfg.points()
+    qs = cfg.queries(q=200)
+    idx = _psb().psb_build(pts, cfg.fanout)
+    exp = oracle.Tree(pts).knn(qs, cfg.k)
+    for algo in ALGOS:
+        assert_same(run(idx, qs, cfg.k, algo), exp, f"C4 {algo}")
+    idx.free()
+
+
+@pytest.mark.parametrize("case", [
+    dict(n=1, d=2, F=32, k=4), dict(n=31, d=3, F=32, k=40), dict(n=33, d=3, F=32, k=33),
+    dict(n=1000, d=1, F=32, k=10), dict(n=5000, d=5, F=64, k=20), dict(n=3000, d=64, F=32, k=9),
+    dict(n=20000, d=4, F=256, k=50), dict(n=20000, d=3, F=512, k=128), dict(n=70000, d=2, F=32, k=7),
+    dict(n=4097, d=16, F=128, k=64), dict(n=1500, d=7, F=128, k=1)])
+def test_edge_shapes(case):
+    rng = np.random.default_rng(case["n"] * 7 + case["d"])
+    pts = (rng.normal(size=(case["n"], case["d"])) * 30).astype(np.float32)
+    qs = (rng.normal(size=(64, case["d"])) * 35).astype(np.float32)
+    idx = _psb().psb_build(pts, case["F"])
+    exp = oracle.knn_bruteforce(pts, qs, case["k"])
+    for algo in ALGOS:
+        assert_same(run(idx, qs, case["k"], algo), exp, f"{case} {algo}")
+    idx.free()
+
+
+@pytest.mark.parametrize("kind", ["lattice", "dups", "identical"])
+def test_tie_heavy(kind):
+    rng = np.random.default_rng(4)
+    if kind == "lattice":
+        g = np.stack(np.meshgrid(np.arange(60), np.arange(60), indexing="ij"), -1).reshape(-1, 2)
+        pts = g.astype(np.float32)
+        qs = rng.integers(0, 60, size=(100, 2)).astype(np.float32)
+    elif kind == "dups":
+        base = rng.integers(0, 5, size=(40, 3)).astype(np.float32)
+        pts = base[rng.integers(0, 40, size=5000)]
+        qs = rng.integers(0, 5, size=(100, 3)).astype(np.float32)
+    else:
+        pts = np.ones((3000, 3), np.float32)
+        qs = rng.normal(size=(50, 3)).astype(np.float32)
+    idx = _psb().psb_build(pts, 32)
+    for k in (1, 13, 64, 128):
+        exp = oracle.knn_bruteforce(pts, qs, k)
+        for algo in ALGOS:
+            assert_same(run(idx, qs, k, algo), exp, f"{kind} k={k} {algo}")
+    idx.free()
+
+
+def test_fma_case_on_gpu():
+    import json, os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "hand_cases.json")))["fma_case"]
+    p = np.array([[float.fromhex(v) for v in g["point"]]] * 40, np.float32)
+    q = np.array([[float.fromhex(v) for v in g["query"]]], np.float32)
+    idx = _psb().psb_build(p, 32)
+    for algo in ALGOS:
+        ids, d = run(idx, q, 1, algo)
+        assert int(d.view(np.uint32)[0, 0]) == int(g["rn_bits"], 16)
+    idx.free()
+
+
+def test_hand_cases_on_gpu():
+    import json, os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "hand_cases.json")))
+    for c in g["cases"]:
+        P = np.array(c["points"], np.float32)
+        idx = _psb().psb_build(P, 32)
+        for algo in ALGOS:
+            ids, d = run(idx, np.array([c["query"]], np.float32), c["k"], algo)
+            assert ids[0].tolist() == c["ids"], (c["name"], algo)
+            assert d[0].tolist() == [float("inf") if v == "inf" else float(v) for v in c["dists"]]
+        idx.free()
+
+
+def test_packing_and_fanout_invariance():
+    cfg = W.config("C2")
+    pts = cfg.points(n=200_000)
+    qs = cfg.queries(q=500)
+    exp = oracle.knn_bruteforce(pts, qs, 32)
+    psb = _psb()
+    for F in (32, 64, 128, 256):
+        for pack in (psb.PSB_PACK_HILBERT, psb.PSB_PACK_STR):
+            idx = psb.psb_build_ex(pts, F, packing=pack)
+            assert_same(run(idx, qs, 32), exp, f"F={F} pack={pack}")
+            idx.free()
+
+
+def test_export_matches_host_blob():
+    psb = _psb()
+    pts = W.gen_uniform(5000, 3, 12)
+    idx = psb.psb_build_ex(pts, 64, id_base=5)
+    a = psb.psb_index_export(idx)
+    b = psb.psb_build_host_blob(pts, 64, id_base=5)
+    assert np.array_equal(a["pts"], b["pts"]) and np.array_equal(a["ids"], b["ids"])
+    for lv in a["nodes"]:
+        assert np.array_equal(a["nodes"][lv], b["nodes"][lv])
+    # device input for psb_build_ex gives the same index
+    idx2 = psb.psb_build_ex(torch.from_numpy(pts).cuda(), 64, id_base=5)
+    c = psb.psb_index_export(idx2)
+    assert np.array_equal(a["pts"], c["pts"]) and np.array_equal(a["ids"], c["ids"])
+    idx.free()
+    idx2.free()
+
+
+def test_data_sharded_merge_equals_unsharded():
+    """Data-sharded mode on one GPU: P sub-trees over slabs (global ids via
+    id_base), local kNN on each, psb_merge_topk -> identical to unsharded/oracle."""
+    psb = _psb()
+    cfg = W.config("C2")
+    pts = cfg.points(n=300_000)
+    qs = cfg.queries(q=2000)
+    exp = oracle.Tree(pts).knn(qs, 32)
+    qd = torch.from_numpy(qs).cuda()
+    for P in (2, 3, 8):
+        bounds = [len(pts) * r // P for r in range(P + 1)]
+        ids = torch.empty((P, len(qs), 32), dtype=torch.int32, device="cuda")
+        ds = torch.empty((P, len(qs), 32), dtype=torch.float32, device="cuda")
+        for r in range(P):
+            sub = psb.psb_build_ex(pts[bounds[r]:bounds[r + 1]], 64, id_base=bounds[r])
+            psb.psb_knn(sub, qd, 32, out=(ids[r], ds[r]))
+            torch.cuda.synchronize()
+            sub.free()
+        mi, md = psb.psb_merge_topk(ids, ds, 32)
+        torch.cuda.synchronize()
+        assert_same((mi.cpu().numpy(), md.cpu().numpy()), exp, f"sharded P={P}")
+
+
+def test_error_codes_on_gpu():
+    psb = _psb()
+    pts = W.gen_uniform(100, 2, 1)
+    idx = psb.psb_build(pts, 32)
+    qd = torch.zeros((4, 2), device="cuda")
+    with pytest.raises(psb.PSBError) as e:
+        psb.psb_knn(idx, qd, 0)
+    assert e.value.code == psb.PSB_EINVAL
+    with pytest.raises(psb.PSBError) as e:
+        psb.psb_knn(idx, qd, 129)
+    assert e.value.code == psb.PSB_EUNSUPPORTED
+    # q = 0 is a no-op
+    ids, d = psb.psb_knn(idx, torch.zeros((0, 2), device="cuda"), 5)
+    assert ids.shape == (0, 5)
+    with pytest.raises(psb.PSBError):
+        psb.psb_build(np.full((10, 2), np.inf, np.float32), 32)
+    idx.free()
