@@ -1,0 +1,377 @@
+#!/usr/bin/env python3
+"""bench.py — PSB exact kNN throughput on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--mode query|data]
+                    [--algo psb|bnb|brute] [--impl ours|reference]
+
+A step is one pass of the whole hot path (one psb_knn
+launch) over one batch of synthetic queries of the named config, inputs resident
+in HBM. N=1 default workload: BASELINE.json configs[1] (C2: 3-D clustered n=1M,
+fanout 64, 10,000 queries, k=32). Multi-GPU (torchrun, one rank per GPU):
+  --mode query (default): replicated index, each rank answers its own batch of
+      q queries (weak scaling, no collective);
+  --mode data: each rank holds a sub-tree over a slab of the points, every rank
+      answers the same q queries, NCCL all-gather + on-device merge (strong).
+L2 is flushed (256 MiB write) between timed steps; each step is timed with CUDA
+events on the launching stream; the reported time is the max over ranks.
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import workloads as W  # noqa: E402
+
+METRIC = "kNN queries/s (PSB exact kNN, batch throughput)"
+UNIT = "queries/s"
+FALLBACK_HBM_GBS = 6650.0
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=300)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--config", default="C2", choices=sorted(W.CONFIGS))
+    ap.add_argument("--queries", type=int, default=0, help="override q per step (0 = config's)")
+    ap.add_argument("--mode", default="query", choices=["query", "data"])
+    ap.add_argument("--algo", default="psb", choices=["psb", "bnb", "brute"])
+    ap.add_argument("--variant", type=int, default=0)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-extras", action="store_true", help="skip latency/e2e/comparator legs")
+    ap.add_argument("--profile", action="store_true", help="short run for ncu (no extras)")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks/throttle sampling DURING the timed region (B200_PROFILING.md)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,utilization.gpu,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index: int):
+        self.dev = device_index
+        self.rows = []
+        self.proc = None
+        self.t = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.dev}", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "50"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+            return
+        self.t = threading.Thread(target=self._read, daemon=True)
+        self.t.start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([c.strip() for c in line.split(",")])
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.12)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        rows = [r for r in self.rows if len(r) >= 9]
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        busy = [float(r[1]) for r in rows if r[4].isdigit() and int(r[4]) > 0] or sm
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(busy) if busy else None,
+                "sm_max_mhz": float(rows[0][2]) if rows[0][2].replace(".", "").isdigit() else None,
+                "reasons": reasons, "samples": len(rows), "samples_busy": len(busy)}
+
+
+# ----------------------------------------------------------------------------- helpers
+def peaks() -> tuple[float, str]:
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        return float(json.load(open(p))["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+def traffic_from_profiles(config: str, algo: str):
+    """dram read+write bytes per launch from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        t = json.load(open(p))
+        return t[f"{config}/{algo}"]["dram_bytes_per_launch"]
+    except Exception:
+        return None
+
+
+def cpu_baseline(cfg, pts, qs, k, gpu_ids=None, gpu_d=None) -> dict:
+    """The oracle as it stands, on this host's cores (bounded sample)."""
+    import oracle
+    threads = os.cpu_count() or 1
+    t0 = time.perf_counter()
+    tree = oracle.Tree(pts)
+    t_build = time.perf_counter() - t0
+    reps = []
+    res = None
+    for _ in range(3):
+        t0 = time.perf_counter()
+        res = tree.knn(qs, k, threads=threads)
+        reps.append(time.perf_counter() - t0)
+    bnb_qps = len(qs) / statistics.median(reps)
+    nb = min(len(qs), 1000 if cfg.n <= 2_000_000 else 100)
+    t0 = time.perf_counter()
+    bf = oracle.knn_bruteforce(pts, qs[:nb], k, threads=threads)
+    bf_qps = nb / (time.perf_counter() - t0)
+    out = {"value": bnb_qps, "unit": UNIT, "cores": threads, "kind": "oracle",
+           "sample": f"all {len(qs)} queries of {cfg.name} via the oracle's recursive B&B (median of 3; "
+                     f"tree build {t_build:.2f}s excluded); brute-force route on {nb} queries",
+           "bruteforce_value": bf_qps,
+           "oracle_routes_agree": bool(np.array_equal(bf[0], res[0][:nb]))}
+    if gpu_ids is not None:
+        out["agrees_with_gpu"] = bool(np.array_equal(gpu_ids, res[0]) and
+                                      np.array_equal(gpu_d.view(np.uint32), res[1].view(np.uint32)))
+    return out
+
+
+# ----------------------------------------------------------------------------- reference arm
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle on the host cores (the tier's reference arm)."""
+    if rank != 0:
+        return
+    import oracle
+    cfg = W.config(args.config)
+    q = args.queries or cfg.q
+    pts = cfg.points()
+    qs = cfg.queries(q)
+    tree = oracle.Tree(pts)
+    threads = os.cpu_count() or 1
+    for _ in range(max(0, args.warmup)):
+        tree.knn(qs[: min(q, 1000)], cfg.k, threads=threads)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        tree.knn(qs, cfg.k, threads=threads)
+        times.append(time.perf_counter() - t0)
+    total = sum(times)
+    val = q * args.steps / total
+    line = {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic (workloads/, seeded)", "impl": "reference",
+            "config": {**cfg.describe(), "q": q, "parallelism": "host threads"},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": threads, "kind": "oracle",
+                             "sample": f"each step: all {q} queries of {cfg.name} via the oracle's "
+                                       f"recursive B&B on {threads} host threads"},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- our arm
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icpp_namkn16_b200 as psb
+    from paper_conf_icpp_namkn16_b200 import dist as pdist
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if args.profile:
+        args.no_extras = True
+        args.no_cpu_baseline = True
+
+    cfg = W.config(args.config)
+    q = args.queries or cfg.q
+    k = cfg.k
+    algo = {"psb": psb.PSB_ALGO_PSB, "bnb": psb.PSB_ALGO_BNB, "brute": psb.PSB_ALGO_BRUTE}[args.algo]
+    pts = cfg.points()
+    if args.mode == "query":
+        # weak scaling: rank r answers its own batch of q queries on a replica
+        all_q = cfg.queries(q * world)
+        qs = all_q[rank * q:(rank + 1) * q]
+        idx = psb.psb_build(pts, cfg.fanout)
+    else:
+        qs = cfg.queries(q)
+        idx = pdist.build_shard(pts, cfg.fanout, world, rank)
+    stream = torch.cuda.current_stream()
+    qd = torch.from_numpy(qs).cuda()
+    out_i = torch.empty((q, k), dtype=torch.int32, device="cuda")
+    out_d = torch.empty((q, k), dtype=torch.float32, device="cuda")
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+
+    # algorithmic bytes of one launch (deterministic traversal counters)
+    if algo == psb.PSB_ALGO_BRUTE:
+        alg_bytes = idx.leaves * idx.fanout * (idx.d * 4) * q + q * (4 * idx.d + 8 * k)
+        stats_sum = None
+    else:
+        _, _, st = psb.psb_knn_stats(idx, qd, k, algo=algo, variant=args.variant, out=(out_i, out_d))
+        stats_sum = st.sum(0).tolist()
+        alg_bytes = psb.algorithmic_bytes(idx, stats_sum, q, k)
+
+    def local_knn(qq, kk):
+        return psb.psb_knn_ex(idx, qq, kk, algo=algo, variant=args.variant,
+                              out=(out_i, out_d) if qq.shape[0] == q else None)
+
+    def step():
+        if args.mode == "query" or world == 1:
+            local_knn(qd, k)
+        else:
+            pdist.data_sharded_knn(local_knn, pdist.device_merge, qd, k)
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+
+    sampler = ClockSampler(local)
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+           for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    sampler.start()
+    time.sleep(0.15)
+    for i in range(args.steps):
+        flush.fill_(i & 0xFF)                      # evict the index from L2 between steps
+        evs[i][0].record(stream)
+        step()
+        evs[i][1].record(stream)
+    torch.cuda.synchronize()
+    clocks = sampler.stop()
+    if world > 1:
+        dist.barrier()
+    step_ms = [a.elapsed_time(b) for a, b in evs]
+    total_ms = torch.tensor([sum(step_ms)], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(total_ms, op=dist.ReduceOp.MAX)
+    total_ms = float(total_ms.item())
+    units = q * world if args.mode == "query" else q
+    value = units * args.steps / (total_ms / 1e3)
+    ms_per_step = total_ms / args.steps
+    kern_s = statistics.mean(step_ms) / 1e3
+    peak, peak_src = peaks()
+    achieved = alg_bytes / kern_s / 1e9
+    traffic = traffic_from_profiles(args.config, args.algo)
+
+    extras = {}
+    if not args.no_extras:
+        # e2e through the public API with HOST (pinned) buffers: H2D + kernel + D2H each step
+        hq = torch.from_numpy(qs).pin_memory()
+        hi = torch.empty((q, k), dtype=torch.int32, pin_memory=True)
+        hd = torch.empty((q, k), dtype=torch.float32, pin_memory=True)
+        e2e_ms = []
+        for i in range(max(3, args.warmup) + args.steps):
+            flush.fill_(i & 0xFF)
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            psb.psb_knn_ex(idx, hq, k, algo=algo, variant=args.variant, out=(hi, hd))
+            stream.synchronize()
+            if i >= max(3, args.warmup):
+                e2e_ms.append((time.perf_counter() - t0) * 1e3)
+        e2e_t = torch.tensor([sum(e2e_ms)], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+        extras["e2e"] = {"value": units * args.steps / (float(e2e_t.item()) / 1e3), "unit": UNIT,
+                         "h2d_bytes_per_step": int(q * idx.d * 4), "d2h_bytes_per_step": int(q * k * 8),
+                         "api": "psb_knn_ex with pinned host buffers (library stages H2D/D2H on the stream)"}
+        if args.mode == "data" and world > 1:
+            extras["e2e"]["note"] = "local search only (the data-sharded all-gather runs on device buffers)"
+        # single-query latency: launch -> results on the host
+        lat = []
+        h1i = torch.empty((1, k), dtype=torch.int32, pin_memory=True)
+        h1d = torch.empty((1, k), dtype=torch.float32, pin_memory=True)
+        nl = min(q, 300)
+        for i in range(nl + 10):
+            h1q = hq[i % q:i % q + 1]
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            psb.psb_knn_ex(idx, h1q, k, algo=algo, variant=args.variant, out=(h1i, h1d))
+            stream.synchronize()
+            if i >= 10:
+                lat.append((time.perf_counter() - t0) * 1e6)
+        lat.sort()
+        extras["latency_us"] = {"p50": lat[len(lat) // 2], "p99": lat[int(len(lat) * 0.99)],
+                                "queries": nl, "definition": "one query per call, launch to results "
+                                "in pinned host memory (PAPER.md L835-838 'query response time')"}
+        # comparators on the same batch (same timing protocol, fewer steps)
+        comp = {}
+        for name, a in (("psb", psb.PSB_ALGO_PSB), ("bnb", psb.PSB_ALGO_BNB), ("brute", psb.PSB_ALGO_BRUTE)):
+            reps = 20 if name != "brute" else 5
+            ts = []
+            for i in range(reps + 2):
+                flush.fill_(i & 0xFF)
+                s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                s.record(stream)
+                psb.psb_knn_ex(idx, qd, k, algo=a, out=(out_i, out_d))
+                e.record(stream)
+                torch.cuda.synchronize()
+                if i >= 2:
+                    ts.append(s.elapsed_time(e))
+            comp[name] = {"queries_per_s": q / (statistics.median(ts) / 1e3), "ms": statistics.median(ts)}
+        extras["comparators_1gpu"] = comp
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        psb.psb_knn_ex(idx, qd, k, algo=algo, variant=args.variant, out=(out_i, out_d))
+        torch.cuda.synchronize()
+        cpu = cpu_baseline(cfg, pts, qs, k, out_i.cpu().numpy(), out_d.cpu().numpy())
+
+    if rank == 0:
+        kernel = {"psb": "psb_kernel", "bnb": "bnb_kernel", "brute": "brute_kernel+merge_kernel"}[args.algo]
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": max(3, args.warmup), "ms_per_step": ms_per_step, "higher_is_better": True,
+            "scaling": "weak" if args.mode == "query" else "strong", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic (workloads/: seeded SplitMix64 uniform / 100-cluster Gaussian)",
+            "config": {**cfg.describe(), "q": q, "algo": args.algo, "variant": args.variant,
+                       "parallelism": (f"query-sharded x{world} (replicated index)" if args.mode == "query"
+                                       else f"data-sharded x{world} (NCCL all-gather + merge)"),
+                       "l2": "flushed between steps (256 MiB write)", "index_bytes": idx.device_bytes},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic, "kernel": kernel,
+                         "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src,
+                         "avg_launch_ms": kern_s * 1e3,
+                         "counters_per_query": (None if stats_sum is None else
+                                                {"node_fetches": stats_sum[0] / q, "leaf_scans": stats_sum[1] / q,
+                                                 "id_loads": stats_sum[2] / q, "cache_hits": stats_sum[3] / q})},
+            "clocks": clocks,
+            "gpu_launches": args.steps * (1 if args.algo != "brute" else 2) * (1 if args.mode == "query" or world == 1 else 2),
+            **extras,
+        }
+        if cpu is not None:
+            line["cpu_baseline"] = cpu
+        print(json.dumps(line), flush=True)
+    idx.free()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

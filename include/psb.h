@@ -21,7 +21,9 @@
  *  - Ids are 0-based input row numbers plus the index's id_base.
  *  - Layouts: points[n][d], queries[q][d] fp32 row-major; out_ids[q][k] int32,
  *    out_dists[q][k] fp32, row-major.
- *  - Pointers to queries/outputs are CUDA device pointers on the index's device
+ *  - Queries and outputs may be CUDA device pointers on the index's device or
+ *    host memory (pinned for asynchronous copies). Host buffers are staged
+ *    through stream-ordered device scratch with cudaMemcpyAsync on `stream`
  *    (psb_build: points may be host or device memory).
  *  - Query calls are asynchronous on `stream` (a cudaStream_t; NULL = legacy
  *    default stream). Argument errors are returned synchronously without
@@ -117,6 +119,18 @@ enum { PSB_VAR_NOCACHE = 1, PSB_VAR_NOMAXDIST = 2 };
 int psb_knn_ex(const psb_index *idx, const float *queries, int64_t q, int32_t k,
                int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant);
 enum { PSB_ALGO_PSB = 0, PSB_ALGO_BNB = 1, PSB_ALGO_BRUTE = 2 };
+
+/* psb_knn_ex (algo PSB_ALGO_PSB or PSB_ALGO_BNB) that also writes per-query
+ * traversal counters to `stats`, a DEVICE array int64[q][4]:
+ *   {internal-node fetches from memory, leaf scans, point ids loaded,
+ *    internal-node visits served by the path cache}.
+ * The counters define the algorithmic bytes of a launch:
+ *   fetches*fanout*2*d*4 + leaf_scans*fanout*d*4 + ids*4 + q*(4*d + 8*k).
+ * The traversal (and hence every counter) is deterministic: a counting run and
+ * a timing run do the same work. Results are identical to psb_knn_ex. */
+int psb_knn_stats(const psb_index *idx, const float *queries, int64_t q, int32_t k,
+                  int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant,
+                  int64_t *stats);
 
 /* Merge `parts` per-shard result sets ids/dists[parts][q][k] (each row ascending
  * by (dist, id), ids global) into the first k of their union, out[q][k]

@@ -30,7 +30,7 @@ FANOUTS = (32, 64, 128, 256, 512)
 
 # every symbol include/psb.h declares (tests check the .so exports all of them)
 EXPORTS = ("psb_build", "psb_build_ex", "psb_knn", "psb_knn_branch_and_bound", "psb_knn_bruteforce",
-           "psb_knn_ex", "psb_merge_topk", "psb_index_info", "psb_index_export", "psb_build_host_blob",
+           "psb_knn_ex", "psb_knn_stats", "psb_merge_topk", "psb_index_info", "psb_index_export", "psb_build_host_blob",
            "psb_free", "psb_last_error", "psb_version")
 
 if not os.path.exists(LIB_PATH):
@@ -47,6 +47,7 @@ _sig = {
     "psb_knn_branch_and_bound": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp]),
     "psb_knn_bruteforce": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp]),
     "psb_knn_ex": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp, _i32, _u32]),
+    "psb_knn_stats": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp, _i32, _u32, _vp]),
     "psb_merge_topk": (ctypes.c_int, [_vp, _vp, _i32, _i64, _i32, _vp, _vp, _vp]),
     "psb_index_info": (ctypes.c_int, [_vp, _P(_i64), _P(_i32), _P(_i32), _P(_i64), _P(_i32), _P(_i64)]),
     "psb_index_export": (ctypes.c_int, [_vp, _vp, _i64, _P(_i64)]),
@@ -153,15 +154,18 @@ def psb_build(points, fanout: int) -> Index:
 
 
 def _query_buffers(index: Index, queries, k: int, out):
+    """Queries: float32 [q, d] tensor on the index's device, or a CPU tensor
+    (pinned for asynchronous copies) — then the library stages it on the stream.
+    Outputs default to the queries' device (CPU outputs are pinned)."""
     torch = _torch()
-    if not (queries.is_cuda and queries.dtype == torch.float32 and queries.dim() == 2
-            and queries.shape[1] == index.d):
-        raise ValueError(f"queries must be a CUDA float32 [q, {index.d}] tensor")
+    if not (queries.dtype == torch.float32 and queries.dim() == 2 and queries.shape[1] == index.d):
+        raise ValueError(f"queries must be a float32 [q, {index.d}] tensor")
     queries = queries.contiguous()
     q = queries.shape[0]
     if out is None:
-        ids = torch.empty((q, k), dtype=torch.int32, device=queries.device)
-        dists = torch.empty((q, k), dtype=torch.float32, device=queries.device)
+        pin = not queries.is_cuda
+        ids = torch.empty((q, k), dtype=torch.int32, device=queries.device, pin_memory=pin)
+        dists = torch.empty((q, k), dtype=torch.float32, device=queries.device, pin_memory=pin)
     else:
         ids, dists = out
     return queries, q, ids, dists
@@ -174,6 +178,26 @@ def psb_knn_ex(index: Index, queries, k: int, algo: int = PSB_ALGO_PSB, variant:
     _check(_lib.psb_knn_ex(index.handle, queries.data_ptr(), q, k, ids.data_ptr(), dists.data_ptr(),
                            _stream_handle(stream), algo, variant), "psb_knn_ex")
     return ids, dists
+
+
+def psb_knn_stats(index: Index, queries, k: int, algo: int = PSB_ALGO_PSB, variant: int = 0,
+                  stream=None, out=None):
+    """psb_knn_ex plus per-query counters: returns (ids, dists, stats int64 [q, 4] on device)
+    with stats = {node fetches, leaf scans, id loads, path-cache hits}."""
+    torch = _torch()
+    queries, q, ids, dists = _query_buffers(index, queries, k, out)
+    stats = torch.zeros((q, 4), dtype=torch.int64, device=f"cuda:{index.device}")
+    _check(_lib.psb_knn_stats(index.handle, queries.data_ptr(), q, k, ids.data_ptr(), dists.data_ptr(),
+                              _stream_handle(stream), algo, variant, stats.data_ptr()), "psb_knn_stats")
+    return ids, dists, stats
+
+
+def algorithmic_bytes(index: Index, stats, q: int, k: int) -> int:
+    """Bytes a launch must move: node blocks fetched, leaf blocks
+    scanned, ids loaded, queries read, results written."""
+    s = stats.sum(0).tolist() if hasattr(stats, "sum") else stats
+    F, d = index.fanout, index.d
+    return int(s[0] * F * 2 * d * 4 + s[1] * F * d * 4 + s[2] * 4 + q * (4 * d + 8 * k))
 
 
 def psb_knn(index: Index, queries, k: int, stream=None, out=None):

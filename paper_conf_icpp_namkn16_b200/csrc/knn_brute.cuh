@@ -1,4 +1,5 @@
-// knn_brute.cu — GPU brute-force kNN (the paper's exhaustive baseline, PAPER.md
+#pragma once
+// knn_brute.cuh — GPU brute-force kNN (the paper's exhaustive baseline, PAPER.md
 // P:L79-84 §I, §V-D) and the k-way merge of sorted per-part lists
 // (data-sharded mode; also the second stage of a chunked scan).
 //
@@ -28,7 +29,8 @@ brute_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k, 
     const int64_t q0 = ((int64_t)blockIdx.x * BF_WARPS + w) * QW;
     if (q0 >= nq) return;
     const int d = ix.d;
-    float *qs = reinterpret_cast<float *>(smem) + (size_t)w * QW * PSB_DMAX;
+    u64 *scratch = reinterpret_cast<u64 *>(smem) + (size_t)w * 32;
+    float *qs = reinterpret_cast<float *>(smem + BF_WARPS * 32 * 8) + (size_t)w * QW * PSB_DMAX;
 
     Query<D> q[QW];
 #pragma unroll
@@ -72,7 +74,7 @@ brute_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k, 
 #pragma unroll
                 for (int t = 0; t < V; ++t)
                     cand[t] = dist[i][t] <= td ? make_key(dist[i][t], __ldg(lid + t)) : ~0ull;
-                T[i].template offer<V>(cand, k, lane, thr[i]);
+                T[i].template offer<V>(cand, k, lane, thr[i], scratch);
             }
         }
     }
@@ -82,47 +84,9 @@ brute_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k, 
         if (q0 + i < nq) T[i].store(k, lane, out_ids + (part + q0 + i) * k, out_dists + (part + q0 + i) * k);
 }
 
-template <int KS>
-__global__ void __launch_bounds__(128)
-merge_kernel(const int32_t *__restrict__ ids, const float *__restrict__ dists, int parts, int64_t nq,
-             int k, int32_t *__restrict__ out_ids, float *__restrict__ out_dists)
-{
-    const int lane = threadIdx.x & 31;
-    const int64_t qi = (int64_t)blockIdx.x * 4 + (threadIdx.x >> 5);
-    if (qi >= nq) return;
-    TopK<KS> T;
-#pragma unroll
-    for (int s = 0; s < KS; ++s) {
-        const int r = s * 32 + lane;
-        T.key[s] = r < k ? make_key(__ldg(dists + qi * k + r), __ldg(ids + qi * k + r)) : PAD_KEY;
-    }
-    u64 thr = T.kth(k);
-    for (int p = 1; p < parts; ++p) {
-        const int64_t row = ((int64_t)p * nq + qi) * k;
-        u64 cand[KS];
-#pragma unroll
-        for (int s = 0; s < KS; ++s) {
-            const int r = s * 32 + lane;
-            cand[s] = r < k ? make_key(__ldg(dists + row + r), __ldg(ids + row + r)) : ~0ull;
-        }
-        T.template offer<KS>(cand, k, lane, thr);
-    }
-    T.store(k, lane, out_ids + qi * k, out_dists + qi * k);
-}
-
-int launch_merge(const int32_t *ids, const float *dists, int parts, int64_t nq, int k, int32_t *oi,
-                 float *od, cudaStream_t st)
-{
-    const unsigned blocks = (unsigned)((nq + 3) / 4);
-    if (k <= 32) merge_kernel<1><<<blocks, 128, 0, st>>>(ids, dists, parts, nq, k, oi, od);
-    else if (k <= 64) merge_kernel<2><<<blocks, 128, 0, st>>>(ids, dists, parts, nq, k, oi, od);
-    else merge_kernel<4><<<blocks, 128, 0, st>>>(ids, dists, parts, nq, k, oi, od);
-    return report_cuda(cudaGetLastError(), "merge kernel launch");
-}
-
 template <int D, int V, int KS>
 static int launch_brute_t(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                          float *od, cudaStream_t st, int sm_count)
+                          float *od, cudaStream_t st, int sm_count, cudaMemPool_t pool)
 {
     constexpr int QW = KS >= 4 ? 2 : 4;
     const int64_t warps_q = (nq + QW - 1) / QW;
@@ -135,13 +99,13 @@ static int launch_brute_t(const DevIndex &ix, const float *queries, int64_t nq, 
     if (S < 1) S = 1;
     const int64_t per = (ix.L + S - 1) / S;
     S = (ix.L + per - 1) / per;
-    const size_t smem = D == 0 ? (size_t)BF_WARPS * QW * PSB_DMAX * 4 : 0;
+    const size_t smem = BF_WARPS * 32 * 8 + (D == 0 ? (size_t)BF_WARPS * QW * PSB_DMAX * 4 : 0);
     int32_t *pi = oi;
     float *pd = od;
     if (S > 1) {
-        cudaError_t e = cudaMallocAsync((void **)&pi, sizeof(int32_t) * (size_t)(S * nq * k), st);
+        cudaError_t e = cudaMallocFromPoolAsync((void **)&pi, sizeof(int32_t) * (size_t)(S * nq * k), pool, st);
         if (e != cudaSuccess) return report_cuda(e, "cudaMallocAsync (brute scratch)");
-        e = cudaMallocAsync((void **)&pd, sizeof(float) * (size_t)(S * nq * k), st);
+        e = cudaMallocFromPoolAsync((void **)&pd, sizeof(float) * (size_t)(S * nq * k), pool, st);
         if (e != cudaSuccess) { cudaFreeAsync(pi, st); return report_cuda(e, "cudaMallocAsync (brute scratch)"); }
     }
     dim3 grid((unsigned)blocks_q, (unsigned)S);
@@ -157,42 +121,28 @@ static int launch_brute_t(const DevIndex &ix, const float *queries, int64_t nq, 
 
 template <int D, int V>
 static int launch_brute_ks(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                           float *od, cudaStream_t st, int sm)
+                           float *od, cudaStream_t st, int sm, cudaMemPool_t pool)
 {
-    if (k <= 32) return launch_brute_t<D, V, 1>(ix, queries, nq, k, oi, od, st, sm);
-    if (k <= 64) return launch_brute_t<D, V, 2>(ix, queries, nq, k, oi, od, st, sm);
-    return launch_brute_t<D, V, 4>(ix, queries, nq, k, oi, od, st, sm);
+    if (k <= 32) return launch_brute_t<D, V, 1>(ix, queries, nq, k, oi, od, st, sm, pool);
+    if (k <= 64) return launch_brute_t<D, V, 2>(ix, queries, nq, k, oi, od, st, sm, pool);
+    return launch_brute_t<D, V, 4>(ix, queries, nq, k, oi, od, st, sm, pool);
 }
 
 template <int D>
-static int launch_brute_v(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                          float *od, cudaStream_t st, int sm)
+int launch_brute_v(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
+                          float *od, cudaStream_t st, int sm, cudaMemPool_t pool)
 {
     switch (ix.F) {
-    case 32: return launch_brute_ks<D, 1>(ix, queries, nq, k, oi, od, st, sm);
-    case 64: return launch_brute_ks<D, 2>(ix, queries, nq, k, oi, od, st, sm);
-    case 128: return launch_brute_ks<D, 4>(ix, queries, nq, k, oi, od, st, sm);
+    case 32: return launch_brute_ks<D, 1>(ix, queries, nq, k, oi, od, st, sm, pool);
+    case 64: return launch_brute_ks<D, 2>(ix, queries, nq, k, oi, od, st, sm, pool);
+    case 128: return launch_brute_ks<D, 4>(ix, queries, nq, k, oi, od, st, sm, pool);
     default: break;
     }
     if constexpr (D == 0) {
-        if (ix.F == 256) return launch_brute_ks<0, 8>(ix, queries, nq, k, oi, od, st, sm);
-        if (ix.F == 512) return launch_brute_ks<0, 16>(ix, queries, nq, k, oi, od, st, sm);
-        return PSB_EUNSUPPORTED;
-    } else {
-        return launch_brute_v<0>(ix, queries, nq, k, oi, od, st, sm);
+        if (ix.F == 256) return launch_brute_ks<0, 8>(ix, queries, nq, k, oi, od, st, sm, pool);
+        if (ix.F == 512) return launch_brute_ks<0, 16>(ix, queries, nq, k, oi, od, st, sm, pool);
     }
-}
-
-int launch_brute(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi, float *od,
-                 cudaStream_t st, int sm_count)
-{
-    switch (ix.d) {
-    case 2: return launch_brute_v<2>(ix, queries, nq, k, oi, od, st, sm_count);
-    case 3: return launch_brute_v<3>(ix, queries, nq, k, oi, od, st, sm_count);
-    case 8: return launch_brute_v<8>(ix, queries, nq, k, oi, od, st, sm_count);
-    case 16: return launch_brute_v<16>(ix, queries, nq, k, oi, od, st, sm_count);
-    default: return launch_brute_v<0>(ix, queries, nq, k, oi, od, st, sm_count);
-    }
+    return PSB_NOT_INSTANTIATED;
 }
 
 }  // namespace psb

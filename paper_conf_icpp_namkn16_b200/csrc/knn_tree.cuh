@@ -1,4 +1,5 @@
-// knn_tree.cu — the two tree traversals on sm_100a, one warp per query:
+#pragma once
+// knn_tree.cuh — the two tree traversals on sm_100a, one warp per query:
 //   psb_kernel : Parallel Scan and Backtrack (Alg. 1, §III)
 //   bnb_kernel : classic branch-and-bound (Roussopoulos [17]) made
 //                stackless with parent links as the paper ran it
@@ -8,13 +9,15 @@
 #include "psb_device.cuh"
 #include "psb_launch.h"
 
+
 namespace psb {
 
 constexpr int WARPS_PER_CTA = 4;
 
 struct WarpState {
     float *cache_md;     // [(H+1)][F] child MINDISTs of the node cached per level
-    int64_t *cache_node; // [(H+1)] node id cached per level (-1 = none)
+    int32_t *cache_node; // [(H+1)] node id cached per level (-1 = none)
+    u64 *scratch;        // [32] top-k merge scratch
     float *qsmem;        // query (D == 0 only)
 };
 
@@ -25,9 +28,11 @@ __device__ __forceinline__ WarpState warp_state(unsigned char *smem, int H, int 
     WarpState s;
     s.cache_md = reinterpret_cast<float *>(base);
     size_t off = (WarpSmem::cache_floats(H, F) * 4 + 15) & ~(size_t)15;
-    s.cache_node = reinterpret_cast<int64_t *>(base + off);
-    off += (size_t)(H + 1) * 8;
+    s.cache_node = reinterpret_cast<int32_t *>(base + off);
+    off += (size_t)(H + 1) * 4;
     off = (off + 15) & ~(size_t)15;
+    s.scratch = reinterpret_cast<u64 *>(base + off);
+    off += 32 * 8;
     s.qsmem = reinterpret_cast<float *>(base + off);
     return s;
 }
@@ -37,7 +42,7 @@ __device__ __forceinline__ WarpState warp_state(unsigned char *smem, int H, int 
 // function of (query, node), and its k-th-MAXDIST bound was applied when it was
 // first fetched (re-applying it could not lower pd further).
 template <int D, int V>
-__device__ __forceinline__ void internal_md(const DevIndex &ix, int lvl, int64_t node,
+__device__ __forceinline__ bool internal_md(const DevIndex &ix, int lvl, int node,
                                             const Query<D> &q, int lane, const WarpState &ws,
                                             bool use_cache, bool use_max, int k, float &pd,
                                             float (&md)[V])
@@ -47,9 +52,9 @@ __device__ __forceinline__ void internal_md(const DevIndex &ix, int lvl, int64_t
     if (use_cache && ws.cache_node[lvl] == node) {
 #pragma unroll
         for (int t = 0; t < V; ++t) md[t] = cm[t];
-        return;
+        return false;
     }
-    const float *blk = ix.nodes + ix.level_off[lvl] + node * ((int64_t)2 * ix.d * F);
+    const float *blk = ix.nodes + ix.level_off[lvl] + (int64_t)node * (2 * ix.d * F);
     float Md[V];
     if (use_max) {
         node_bounds<D, V, true>(blk, q, ix.d, lane, md, Md);
@@ -64,18 +69,38 @@ __device__ __forceinline__ void internal_md(const DevIndex &ix, int lvl, int64_t
         if (lane == 0) ws.cache_node[lvl] = node;
         __syncwarp();
     }
+    return true;
 }
 
-__device__ __forceinline__ int64_t max_leaf(const DevIndex &ix, int lvl, int64_t node)
+// Per-query traversal counters (psb_knn_stats): they define the algorithmic
+// bytes of SURVEY.md §8(d) without changing the traversal.
+struct Stats {
+    uint32_t fetch = 0, hit = 0, leaf = 0, ids = 0;
+    __device__ __forceinline__ void node(bool fetched) { fetched ? ++fetch : ++hit; }
+    __device__ __forceinline__ void write(int64_t *st, int64_t qi, int lane) const
+    {
+        if (st && lane == 0) {
+            st[qi * 4 + 0] = fetch;
+            st[qi * 4 + 1] = leaf;
+            st[qi * 4 + 2] = ids;
+            st[qi * 4 + 3] = hit;
+        }
+    }
+};
+
+// Last leaf under (lvl, node): min((node+1)*F^lvl, L) - 1. With span clamped at
+// L and node < F*nlev[lvl], the product stays below 2L < 2^27 (n < 2^31, F >= 32).
+__device__ __forceinline__ int max_leaf(const DevIndex &ix, int lvl, int node)
 {
-    const int64_t e = (node + 1) * ix.span[lvl];
-    return (e < ix.L ? e : ix.L) - 1;
+    const int e = (node + 1) * (int)ix.span[lvl];
+    return (e < (int)ix.L ? e : (int)ix.L) - 1;
 }
 
 template <int D, int V, int KS>
 __global__ void __launch_bounds__(WARPS_PER_CTA * 32)
 psb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
-           int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant)
+           int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant,
+           int64_t *__restrict__ stats)
 {
     constexpr int F = 32 * V;
     extern __shared__ __align__(16) unsigned char smem[];
@@ -96,15 +121,16 @@ psb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
     T.init();
     u64 thr = PAD_KEY;
     float pd = __int_as_float(0x7f800000);
+    Stats S;
 
     // S2: pass 1, getInitialPruningDistance(Q, ClosestLeaf) (Alg. 1 l.3; R4):
     // greedy descent by (MINDIST, child index) argmin, k-th-MAXDIST bounds on the way.
     int lvl = H;
-    int64_t node = 0;
+    int node = 0;
     while (lvl > 0) {
         float md[V];
-        internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
-        const int64_t base = node * F, nb = ix.nlev[lvl - 1];
+        S.node(internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
+        const int base = node * F, nb = (int)ix.nlev[lvl - 1];
         u64 best = ~0ull;
 #pragma unroll
         for (int t = 0; t < V; ++t) {
@@ -115,17 +141,19 @@ psb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
             }
         }
         best = warp_min_u64(best);
-        node = base + (int64_t)(best & 0xffffffffu);
+        node = base + (int)(best & 0xffffffffu);
         --lvl;
     }
     // ClosestLeaf and its right siblings until k points are seen; their points go
     // straight into the kNN list (allowed by R4: pass 2 then skips these leaves).
-    const int64_t pass1_lo = node;
-    int64_t pass1_hi = node - 1, seen = 0;
-    while (seen < k && pass1_hi + 1 < ix.L) {
+    const int pass1_lo = node;
+    int pass1_hi = node - 1;
+    int64_t seen = 0;
+    while (seen < k && pass1_hi + 1 < (int)ix.L) {
         ++pass1_hi;
-        scan_leaf<D, V, KS>(ix, pass1_hi, q, lane, T, k, thr);
-        const int64_t left = ix.n - pass1_hi * F;
+        scan_leaf<D, V, KS>(ix, pass1_hi, q, lane, T, k, thr, S.ids, ws.scratch);
+        ++S.leaf;
+        const int64_t left = ix.n - (int64_t)pass1_hi * F;
         seen += left < F ? left : F;
     }
     pd = fminf(pd, key_dist(thr));
@@ -134,17 +162,17 @@ psb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
     // parent-link backtrack.
     lvl = H;
     node = 0;
-    int64_t visited = -1;                                        // R10
+    int visited = -1;                                            // R10
     while (true) {
         if (lvl > 0) {
             float md[V];
-            internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
+            S.node(internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
             // S6: eligible(c) = MINDIST <= pd (R5) and unvisited leaves below (R8)
-            const int64_t base = node * F, nb = ix.nlev[lvl - 1];
+            const int base = node * F, nb = (int)ix.nlev[lvl - 1];
             unsigned mine = 0;
 #pragma unroll
             for (int t = 0; t < V; ++t) {
-                const int64_t g = base + lane * V + t;
+                const int g = base + lane * V + t;
                 const bool e = g < nb && md[t] <= pd && max_leaf(ix, lvl - 1, g) > visited;
                 mine |= (unsigned)e << t;
             }
@@ -162,16 +190,17 @@ psb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
             }
         } else {
             // S8-S10: leaf j
-            const int64_t j = node;
+            const int j = node;
             bool changed;
             if (j >= pass1_lo && j <= pass1_hi) {
                 changed = true;                                  // already offered in pass 1
             } else {
-                changed = scan_leaf<D, V, KS>(ix, j, q, lane, T, k, thr);
+                changed = scan_leaf<D, V, KS>(ix, j, q, lane, T, k, thr, S.ids, ws.scratch);
+                ++S.leaf;
             }
             pd = fminf(pd, key_dist(thr));                       // Alg. 1 l.37
             visited = j;                                         // l.38
-            if (j == ix.L - 1) break;                            // R10
+            if (j == (int)ix.L - 1) break;                       // R10
             if (changed) {
                 node = j + 1;                                    // l.41 right sibling (R11, R12)
             } else {
@@ -182,6 +211,7 @@ psb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
     }
     // S11
     T.store(k, lane, out_ids + qi * k, out_dists + qi * k);
+    S.write(stats, qi, lane);
 }
 
 // Stackless B&B: at an internal node take the next child in
@@ -190,7 +220,8 @@ psb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
 template <int D, int V, int KS>
 __global__ void __launch_bounds__(WARPS_PER_CTA * 32)
 bnb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
-           int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant)
+           int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant,
+           int64_t *__restrict__ stats)
 {
     constexpr int F = 32 * V;
     extern __shared__ __align__(16) unsigned char smem[];
@@ -210,14 +241,15 @@ bnb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
     T.init();
     u64 thr = PAD_KEY;
     float pd = __int_as_float(0x7f800000);
+    Stats S;
 
     int lvl = H;
-    int64_t node = 0;
+    int node = 0;
     int from_c = -1;                        // child we returned from, -1 = fresh visit
     while (true) {
         if (lvl > 0) {
             float md[V];
-            internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
+            S.node(internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
             u64 from_key = 0;
             if (from_c >= 0) {
                 float v = md[0];
@@ -226,7 +258,7 @@ bnb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
                     if (t == from_c % V) v = md[t];
                 from_key = make_key(__shfl_sync(FULL, v, from_c / V), from_c);
             }
-            const int64_t base = node * F, nb = ix.nlev[lvl - 1];
+            const int base = node * F, nb = (int)ix.nlev[lvl - 1];
             u64 best = ~0ull;
 #pragma unroll
             for (int t = 0; t < V; ++t) {
@@ -237,7 +269,7 @@ bnb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
             }
             best = warp_min_u64(best);
             if (best != ~0ull) {
-                node = base + (int64_t)(best & 0xffffffffu);
+                node = base + (int)(best & 0xffffffffu);
                 --lvl;
                 from_c = -1;
             } else {
@@ -247,7 +279,8 @@ bnb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
                 ++lvl;
             }
         } else {
-            scan_leaf<D, V, KS>(ix, node, q, lane, T, k, thr);
+            scan_leaf<D, V, KS>(ix, node, q, lane, T, k, thr, S.ids, ws.scratch);
+            ++S.leaf;
             pd = fminf(pd, key_dist(thr));
             from_c = (int)(node % F);
             node /= F;
@@ -255,11 +288,12 @@ bnb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
         }
     }
     T.store(k, lane, out_ids + qi * k, out_dists + qi * k);
+    S.write(stats, qi, lane);
 }
 
 template <int D, int V, int KS>
 static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
-                         int32_t *oi, float *od, cudaStream_t st, uint32_t variant)
+                         int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats)
 {
     const size_t smem = WARPS_PER_CTA * WarpSmem::bytes(ix.H, 32 * V, D == 0);
     const int64_t blocks = (nq + WARPS_PER_CTA - 1) / WARPS_PER_CTA;
@@ -268,48 +302,34 @@ static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return report_cuda(e, "cudaFuncSetAttribute");
     }
-    kern<<<(unsigned)blocks, WARPS_PER_CTA * 32, smem, st>>>(ix, queries, nq, k, oi, od, variant);
+    kern<<<(unsigned)blocks, WARPS_PER_CTA * 32, smem, st>>>(ix, queries, nq, k, oi, od, variant, stats);
     return report_cuda(cudaGetLastError(), "tree kernel launch");
 }
 
 template <int D, int V>
 static int launch_tree_ks(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
-                          int32_t *oi, float *od, cudaStream_t st, uint32_t variant)
+                          int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats)
 {
-    if (k <= 32) return launch_tree_t<D, V, 1>(algo, ix, queries, nq, k, oi, od, st, variant);
-    if (k <= 64) return launch_tree_t<D, V, 2>(algo, ix, queries, nq, k, oi, od, st, variant);
-    return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant);
+    if (k <= 32) return launch_tree_t<D, V, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
+    if (k <= 64) return launch_tree_t<D, V, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
+    return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
 }
 
 template <int D>
-static int launch_tree_v(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
-                         int32_t *oi, float *od, cudaStream_t st, uint32_t variant)
+int launch_tree_v(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
+                         int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats)
 {
     switch (ix.F) {
-    case 32: return launch_tree_ks<D, 1>(algo, ix, queries, nq, k, oi, od, st, variant);
-    case 64: return launch_tree_ks<D, 2>(algo, ix, queries, nq, k, oi, od, st, variant);
-    case 128: return launch_tree_ks<D, 4>(algo, ix, queries, nq, k, oi, od, st, variant);
+    case 32: return launch_tree_ks<D, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
+    case 64: return launch_tree_ks<D, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
+    case 128: return launch_tree_ks<D, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
     default: break;
     }
     if constexpr (D == 0) {
-        if (ix.F == 256) return launch_tree_ks<0, 8>(algo, ix, queries, nq, k, oi, od, st, variant);
-        if (ix.F == 512) return launch_tree_ks<0, 16>(algo, ix, queries, nq, k, oi, od, st, variant);
-        return PSB_EUNSUPPORTED;
-    } else {
-        return launch_tree_v<0>(algo, ix, queries, nq, k, oi, od, st, variant);
+        if (ix.F == 256) return launch_tree_ks<0, 8>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
+        if (ix.F == 512) return launch_tree_ks<0, 16>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
     }
-}
-
-int launch_tree(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                float *od, cudaStream_t st, uint32_t variant)
-{
-    switch (ix.d) {
-    case 2: return launch_tree_v<2>(algo, ix, queries, nq, k, oi, od, st, variant);
-    case 3: return launch_tree_v<3>(algo, ix, queries, nq, k, oi, od, st, variant);
-    case 8: return launch_tree_v<8>(algo, ix, queries, nq, k, oi, od, st, variant);
-    case 16: return launch_tree_v<16>(algo, ix, queries, nq, k, oi, od, st, variant);
-    default: return launch_tree_v<0>(algo, ix, queries, nq, k, oi, od, st, variant);
-    }
+    return PSB_NOT_INSTANTIATED;   // caller falls back to the generic-d kernels
 }
 
 }  // namespace psb

@@ -47,6 +47,7 @@ struct psb_index {
     int32_t *ids = nullptr;
     float *nodes = nullptr;
     int64_t device_bytes = 0;
+    cudaMemPool_t pool = nullptr;   // stream-ordered scratch (host-buffer staging, brute-force partials)
 };
 
 static void index_release(psb_index *ix)
@@ -58,6 +59,7 @@ static void index_release(psb_index *ix)
     cudaFree(ix->pts);
     cudaFree(ix->ids);
     cudaFree(ix->nodes);
+    if (ix->pool) cudaMemPoolDestroy(ix->pool);
     if (prev >= 0) cudaSetDevice(prev);
     delete ix;
 }
@@ -149,6 +151,21 @@ int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int6
         return rc;
     }
     ix->device_bytes = (int64_t)(bp + bi + bn);
+    // Own pool for per-call scratch; memory stays mapped between calls (a zero
+    // release threshold would unmap and remap it at every synchronisation).
+    cudaMemPoolProps props;
+    memset(&props, 0, sizeof props);
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    if ((e = cudaMemPoolCreate(&ix->pool, &props)) != cudaSuccess) {
+        rc = report_cuda(e, "psb_build_ex: cudaMemPoolCreate");
+        ix->pool = nullptr;
+        index_release(ix);
+        return rc;
+    }
+    uint64_t keep = UINT64_MAX;
+    cudaMemPoolSetAttribute(ix->pool, cudaMemPoolAttrReleaseThreshold, &keep);
     *out = ix;
     return PSB_OK;
 }
@@ -180,43 +197,111 @@ static int check_query_args(const char *fn, const psb_index *ix, const float *qu
     return PSB_OK;
 }
 
-int psb_knn_ex(const psb_index *ix, const float *queries, int64_t q, int32_t k, int32_t *out_ids,
-               float *out_dists, void *stream, int32_t algo, uint32_t variant)
+static bool is_device_ptr(const void *p)
+{
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+// Launch one algorithm on device buffers; host buffers (pinned or pageable) are
+// staged through stream-ordered device scratch with copies on the same stream.
+static int knn_impl(const char *fn, const psb_index *ix, const float *queries, int64_t q, int32_t k,
+                    int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant,
+                    int64_t *stats)
 {
     g_err[0] = 0;
-    int rc = check_query_args("psb_knn", ix, queries, q, k, out_ids, out_dists);
+    int rc = check_query_args(fn, ix, queries, q, k, out_ids, out_dists);
     if (rc != PSB_OK) return rc;
     if (variant & ~(uint32_t)(PSB_VAR_NOCACHE | PSB_VAR_NOMAXDIST)) {
-        psb_set_error("psb_knn_ex: unknown variant bits 0x%x", variant);
+        psb_set_error("%s: unknown variant bits 0x%x", fn, variant);
+        return PSB_EINVAL;
+    }
+    if (algo != PSB_ALGO_PSB && algo != PSB_ALGO_BNB && algo != PSB_ALGO_BRUTE) {
+        psb_set_error("%s: unknown algo %d", fn, algo);
+        return PSB_EINVAL;
+    }
+    if (stats && algo == PSB_ALGO_BRUTE) {
+        psb_set_error("%s: stats are defined for the tree traversals only", fn);
         return PSB_EINVAL;
     }
     if (q == 0) return PSB_OK;
-    const DevIndex v = dev_view(ix);
     cudaStream_t st = (cudaStream_t)stream;
-    switch (algo) {
-    case PSB_ALGO_PSB:
-    case PSB_ALGO_BNB: return psb::launch_tree(algo, v, queries, q, k, out_ids, out_dists, st, variant);
-    case PSB_ALGO_BRUTE: return psb::launch_brute(v, queries, q, k, out_ids, out_dists, st, ix->sm_count);
-    default: psb_set_error("psb_knn_ex: unknown algo %d", algo); return PSB_EINVAL;
+    const bool hq = !is_device_ptr(queries);
+    const bool ho = !is_device_ptr(out_ids) || !is_device_ptr(out_dists);
+    const float *dq = queries;
+    int32_t *di = out_ids;
+    float *dd = out_dists;
+    cudaError_t e = cudaSuccess;
+    const size_t bq = sizeof(float) * (size_t)(q * ix->d), bo = sizeof(float) * (size_t)(q * k);
+    if (hq) {
+        float *tmp = nullptr;
+        if ((e = cudaMallocFromPoolAsync((void **)&tmp, bq, ix->pool, st)) != cudaSuccess) return report_cuda(e, fn);
+        if ((e = cudaMemcpyAsync(tmp, queries, bq, cudaMemcpyHostToDevice, st)) != cudaSuccess) {
+            cudaFreeAsync(tmp, st);
+            return report_cuda(e, fn);
+        }
+        dq = tmp;
     }
+    if (ho) {
+        if ((e = cudaMallocFromPoolAsync((void **)&di, bo, ix->pool, st)) != cudaSuccess ||
+            (e = cudaMallocFromPoolAsync((void **)&dd, bo, ix->pool, st)) != cudaSuccess)
+            rc = report_cuda(e, fn);
+    }
+    if (rc == PSB_OK) {
+        const DevIndex v = dev_view(ix);
+        rc = algo == PSB_ALGO_BRUTE ? psb::launch_brute(v, dq, q, k, di, dd, st, ix->sm_count, ix->pool)
+                                    : psb::launch_tree(algo, v, dq, q, k, di, dd, st, variant, stats);
+    }
+    if (ho) {
+        if (rc == PSB_OK && ((e = cudaMemcpyAsync(out_ids, di, bo, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||
+                             (e = cudaMemcpyAsync(out_dists, dd, bo, cudaMemcpyDeviceToHost, st)) != cudaSuccess))
+            rc = report_cuda(e, fn);
+        if (di != out_ids) cudaFreeAsync(di, st);
+        if (dd != out_dists) cudaFreeAsync(dd, st);
+    }
+    if (hq) cudaFreeAsync((void *)dq, st);
+    return rc;
+}
+
+int psb_knn_ex(const psb_index *ix, const float *queries, int64_t q, int32_t k, int32_t *out_ids,
+               float *out_dists, void *stream, int32_t algo, uint32_t variant)
+{
+    return knn_impl("psb_knn_ex", ix, queries, q, k, out_ids, out_dists, stream, algo, variant, nullptr);
+}
+
+int psb_knn_stats(const psb_index *ix, const float *queries, int64_t q, int32_t k, int32_t *out_ids,
+                  float *out_dists, void *stream, int32_t algo, uint32_t variant, int64_t *stats)
+{
+    if (!stats && q > 0) { psb_set_error("psb_knn_stats: stats is NULL"); return PSB_EINVAL; }
+    if (stats && q > 0 && !is_device_ptr(stats)) {
+        psb_set_error("psb_knn_stats: stats must be device memory");
+        return PSB_EINVAL;
+    }
+    return knn_impl("psb_knn_stats", ix, queries, q, k, out_ids, out_dists, stream, algo, variant, stats);
 }
 
 int psb_knn(const psb_index *ix, const float *queries, int64_t q, int32_t k, int32_t *out_ids,
             float *out_dists, void *stream)
 {
-    return psb_knn_ex(ix, queries, q, k, out_ids, out_dists, stream, PSB_ALGO_PSB, 0);
+    return knn_impl("psb_knn", ix, queries, q, k, out_ids, out_dists, stream, PSB_ALGO_PSB, 0, nullptr);
 }
 
 int psb_knn_branch_and_bound(const psb_index *ix, const float *queries, int64_t q, int32_t k,
                              int32_t *out_ids, float *out_dists, void *stream)
 {
-    return psb_knn_ex(ix, queries, q, k, out_ids, out_dists, stream, PSB_ALGO_BNB, 0);
+    return knn_impl("psb_knn_branch_and_bound", ix, queries, q, k, out_ids, out_dists, stream, PSB_ALGO_BNB,
+                    0, nullptr);
 }
 
 int psb_knn_bruteforce(const psb_index *ix, const float *queries, int64_t q, int32_t k,
                        int32_t *out_ids, float *out_dists, void *stream)
 {
-    return psb_knn_ex(ix, queries, q, k, out_ids, out_dists, stream, PSB_ALGO_BRUTE, 0);
+    return knn_impl("psb_knn_bruteforce", ix, queries, q, k, out_ids, out_dists, stream, PSB_ALGO_BRUTE,
+                    0, nullptr);
 }
 
 int psb_merge_topk(const int32_t *ids, const float *dists, int32_t parts, int64_t q, int32_t k,

@@ -176,6 +176,30 @@ __device__ __forceinline__ float kth_bound(const float (&Md)[V], int k, float pd
     return __uint_as_float(res);
 }
 
+// Warp bitonic network on one u64 key per lane: sort ascending by lane, and the
+// final merge stage alone (a bitonic sequence -> ascending).
+__device__ __forceinline__ u64 cmpx(u64 v, int j, bool take_min)
+{
+    const u64 o = __shfl_xor_sync(FULL, v, j);
+    return take_min ? (o < v ? o : v) : (o < v ? v : o);
+}
+__device__ __forceinline__ u64 warp_sort32(u64 v, int lane)
+{
+#pragma unroll
+    for (int kk = 2; kk <= 32; kk <<= 1) {
+        const bool asc = (lane & kk) == 0;
+#pragma unroll
+        for (int j = kk >> 1; j > 0; j >>= 1) v = cmpx(v, j, ((lane & j) == 0) == asc);
+    }
+    return v;
+}
+__device__ __forceinline__ u64 warp_merge32(u64 v, int lane)
+{
+#pragma unroll
+    for (int j = 16; j > 0; j >>= 1) v = cmpx(v, j, (lane & j) == 0);
+    return v;
+}
+
 // Warp-distributed sorted top-k of u64 keys (S9; the paper keeps "the kNN list
 // and k pruning distances" in shared memory; here they live in
 // registers): position r = s*32 + lane holds the r-th smallest key, KS keys per
@@ -218,27 +242,78 @@ struct TopK {
             key[s] = r > p ? prev[s] : (r == p ? x : key[s]);
         }
     }
-    // Offer this lane's V candidate keys (~0 = none); returns whether any entered
-    // the first k positions. `thr` is the k-th key, kept current.
-    template <int V>
-    __device__ __forceinline__ bool offer(const u64 (&cand)[V], int k, int lane, u64 &thr)
+    // Merge 32 candidate keys (one per lane, ~0 = none) into the list: sort them
+    // with a warp bitonic network, then for each 32-key segment of the list take
+    // the elementwise min/max against the reversed candidates (the 32 smallest /
+    // largest of the union, each a bitonic sequence) and re-sort both halves;
+    // the larger half carries into the next segment, the last one is dropped.
+    __device__ __forceinline__ void merge32(u64 c, int lane)
     {
-        bool changed = false;
+        c = warp_sort32(c, lane);
+#pragma unroll
+        for (int s = 0; s < KS; ++s) {
+            const u64 rc = __shfl_sync(FULL, c, 31 - lane);
+            const u64 lo = rc < key[s] ? rc : key[s];
+            const u64 hi = rc < key[s] ? key[s] : rc;
+            key[s] = warp_merge32(lo, lane);
+            if (s + 1 < KS) c = warp_merge32(hi, lane);
+        }
+    }
+    // Offer this lane's V candidate keys (~0 = none); returns whether any entered
+    // the first k positions. `thr` is the k-th key, kept current. Few candidates
+    // are inserted one by one; more are compacted through `scratch` (32 u64 of
+    // per-warp shared memory) and merged 32 at a time.
+    template <int V>
+    __device__ __forceinline__ bool offer(const u64 (&cand)[V], int k, int lane, u64 &thr, u64 *scratch)
+    {
+        unsigned bal[V];
+        int m = 0;
 #pragma unroll
         for (int t = 0; t < V; ++t) {
-            unsigned m = __ballot_sync(FULL, cand[t] < thr);
-            while (m) {
-                const int src = __ffs(m) - 1;
-                m &= m - 1;
-                const u64 x = __shfl_sync(FULL, cand[t], src);
-                if (x < thr) {
-                    insert(x, lane);
+            bal[t] = __ballot_sync(FULL, cand[t] < thr);
+            m += __popc(bal[t]);
+        }
+        if (m == 0) return false;
+        if (m <= 2) {
+#pragma unroll
+            for (int t = 0; t < V; ++t) {
+                unsigned b = bal[t];
+                while (b) {
+                    const int src = __ffs(b) - 1;
+                    b &= b - 1;
+                    const u64 x = __shfl_sync(FULL, cand[t], src);
+                    if (x < thr) {
+                        insert(x, lane);
+                        thr = kth(k);
+                    }
+                }
+            }
+            return true;
+        }
+        if (m <= 32) {
+            const unsigned lt = (1u << lane) - 1;
+            int base = 0;
+#pragma unroll
+            for (int t = 0; t < V; ++t) {
+                if (bal[t] >> lane & 1u) scratch[base + __popc(bal[t] & lt)] = cand[t];
+                base += __popc(bal[t]);
+            }
+            __syncwarp();
+            const u64 c = lane < m ? scratch[lane] : ~0ull;
+            __syncwarp();
+            merge32(c, lane);
+        } else {
+#pragma unroll
+            for (int t = 0; t < V; ++t) {
+                const u64 c = cand[t] < thr ? cand[t] : ~0ull;
+                if (__any_sync(FULL, c != ~0ull)) {
+                    merge32(c, lane);
                     thr = kth(k);
-                    changed = true;
                 }
             }
         }
-        return changed;
+        thr = kth(k);
+        return true;
     }
     __device__ __forceinline__ void store(int k, int lane, int32_t *__restrict__ oi,
                                           float *__restrict__ od) const
@@ -257,22 +332,28 @@ struct TopK {
 // S8+S9: scan one leaf, offer its points. Ids are fetched lazily, only for
 // points whose distance can enter the list (dist <= current k-th distance).
 template <int D, int V, int KS>
-__device__ __forceinline__ bool scan_leaf(const DevIndex &ix, int64_t leaf, const Query<D> &q,
-                                          int lane, TopK<KS> &T, int k, u64 &thr)
+__device__ __forceinline__ bool scan_leaf(const DevIndex &ix, int leaf, const Query<D> &q,
+                                          int lane, TopK<KS> &T, int k, u64 &thr, uint32_t &n_ids,
+                                          u64 *scratch)
 {
     constexpr int F = 32 * V;
     float dist[V];
-    leaf_dists<D, V>(ix.pts + leaf * (int64_t)ix.d * F, q, ix.d, lane, dist);
+    leaf_dists<D, V>(ix.pts + (int64_t)leaf * ix.d * F, q, ix.d, lane, dist);
     const float td = key_dist(thr);
     bool any = false;
 #pragma unroll
     for (int t = 0; t < V; ++t) any |= dist[t] <= td;
     if (!__any_sync(FULL, any)) return false;
-    const int32_t *__restrict__ lid = ix.ids + leaf * F + lane * V;
+    const int32_t *__restrict__ lid = ix.ids + (int64_t)leaf * F + lane * V;
     u64 cand[V];
+    int loads = 0;
 #pragma unroll
-    for (int t = 0; t < V; ++t) cand[t] = dist[t] <= td ? make_key(dist[t], __ldg(lid + t)) : ~0ull;
-    return T.template offer<V>(cand, k, lane, thr);
+    for (int t = 0; t < V; ++t) {
+        cand[t] = dist[t] <= td ? make_key(dist[t], __ldg(lid + t)) : ~0ull;
+        loads += dist[t] <= td;
+    }
+    n_ids += __reduce_add_sync(FULL, loads);
+    return T.template offer<V>(cand, k, lane, thr, scratch);
 }
 
 // Per-warp shared-memory layout for the traversal kernels.
@@ -282,8 +363,9 @@ struct WarpSmem {
     {
         size_t b = cache_floats(H, F) * 4;
         b = (b + 15) & ~(size_t)15;
-        b += (size_t)(H + 1) * 8;
+        b += (size_t)(H + 1) * 4;
         b = (b + 15) & ~(size_t)15;
+        b += 32 * 8;                        // top-k merge scratch
         if (qsmem) b += PSB_DMAX * 4;
         return b;
     }

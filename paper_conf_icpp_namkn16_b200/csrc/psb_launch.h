@@ -10,14 +10,26 @@ namespace psb {
 int report_cuda(cudaError_t e, const char *what);
 
 // PSB_ALGO_PSB or PSB_ALGO_BNB, one warp per query (knn_tree.cu).
+// `stats` (nullable, device [nq][4] int64): per query {internal node fetches,
+// leaf scans, id loads, path-cache hits}.
 int launch_tree(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                float *od, cudaStream_t st, uint32_t variant);
+                float *od, cudaStream_t st, uint32_t variant, int64_t *stats);
 
 // Exhaustive scan of all points (knn_brute.cu). Splits the point set into
 // chunks when there are too few queries to fill the GPU and merges the partial
 // lists with launch_merge; scratch is stream-ordered.
 int launch_brute(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi, float *od,
-                 cudaStream_t st, int sm_count);
+                 cudaStream_t st, int sm_count, cudaMemPool_t pool);
+
+// Per-d launchers (instantiated in knn_tree_d*.cu / knn_brute_d*.cu); they
+// return PSB_NOT_INSTANTIATED when (d, fanout) needs the generic-d kernels.
+constexpr int PSB_NOT_INSTANTIATED = 1;
+template <int D>
+int launch_tree_v(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
+                  float *od, cudaStream_t st, uint32_t variant, int64_t *stats);
+template <int D>
+int launch_brute_v(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi, float *od,
+                   cudaStream_t st, int sm, cudaMemPool_t pool);
 
 // [parts][nq][k] sorted (dist, id) lists -> first k of their union (knn_brute.cu).
 int launch_merge(const int32_t *ids, const float *dists, int parts, int64_t nq, int k, int32_t *oi,

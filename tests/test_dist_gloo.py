@@ -1,0 +1,93 @@
+"""Multi-process (world_size 2, gloo on CPU) tests of the multi-GPU host logic in
+paper_conf_icpp_namkn16_b200/dist.py. The local search and merge steps are
+injected (the oracle here; libpsb.so's kernels on GPUs), so what is tested is
+the sharding, id_base bookkeeping, all-gather layout and slice ownership."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import oracle
+import workloads as W
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _np_merge(gi, gd, k):
+    """Reference merge of [parts, q, k] lists by (dist, id) (test helper)."""
+    gi, gd = gi.numpy(), gd.numpy()
+    P, q, _ = gi.shape
+    oi = np.empty((q, k), np.int32)
+    od = np.empty((q, k), np.float32)
+    for r in range(q):
+        pairs = sorted(zip(gd[:, r].ravel().tolist(), gi[:, r].ravel().tolist()),
+                       key=lambda t: (t[0], t[1] if t[1] >= 0 else 2 ** 31))[:k]
+        oi[r] = [p[1] for p in pairs]
+        od[r] = [p[0] for p in pairs]
+    return torch.from_numpy(oi), torch.from_numpy(od)
+
+
+def _worker(rank, world, port, mode, out):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_icpp_namkn16_b200 import dist as pd
+    cfg = W.config("C2")
+    pts = cfg.points(n=20_000)
+    qs = torch.from_numpy(cfg.queries(q=300))
+    k = 16
+    if mode == "data":
+        b = pd.shard_bounds(len(pts), world)
+        slab = pts[b[rank]:b[rank + 1]]
+
+        def local(q, kk):
+            ids, d = oracle.knn_bruteforce(slab, q.numpy(), kk)
+            ids = np.where(ids >= 0, ids + b[rank], -1).astype(np.int32)   # global ids (id_base)
+            return torch.from_numpy(ids), torch.from_numpy(d)
+
+        ids, d = pd.data_sharded_knn(local, _np_merge, qs, k)
+        sl = pd.query_slice(len(qs), world, rank)
+        exp = oracle.knn_bruteforce(pts, qs.numpy()[sl], k)
+        ok = np.array_equal(ids.numpy(), exp[0]) and np.array_equal(d.numpy().view(np.uint32),
+                                                                     exp[1].view(np.uint32))
+        ids2, d2 = pd.data_sharded_knn(local, _np_merge, qs, k, merge_all=True)
+        exp2 = oracle.knn_bruteforce(pts, qs.numpy(), k)
+        ok = ok and np.array_equal(ids2.numpy(), exp2[0])
+    else:
+        def local(q, kk):
+            ids, d = oracle.knn_bruteforce(pts, q.numpy(), kk)
+            return torch.from_numpy(ids), torch.from_numpy(d)
+
+        ids, d = pd.query_sharded_knn(local, qs, k, gather=True)
+        exp = oracle.knn_bruteforce(pts, qs.numpy(), k)
+        ok = np.array_equal(ids.numpy(), exp[0]) and np.array_equal(d.numpy(), exp[1])
+    out[rank] = bool(ok)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("mode", ["data", "query"])
+def test_two_rank_modes(mode):
+    mgr = mp.Manager()
+    out = mgr.dict()
+    mp.spawn(_worker, args=(2, _free_port(), mode, out), nprocs=2, join=True)
+    assert dict(out) == {0: True, 1: True}
+
+
+def test_shard_bounds_cover_exactly():
+    from paper_conf_icpp_namkn16_b200 import dist as pd
+    for n in (1, 7, 10_000, 512_000_000):
+        for w in (1, 2, 3, 8):
+            b = pd.shard_bounds(n, w)
+            assert b[0] == 0 and b[-1] == n and all(b[i] <= b[i + 1] for i in range(w))
+            sizes = [b[i + 1] - b[i] for i in range(w)]
+            assert max(sizes) - min(sizes) <= 1

@@ -268,3 +268,39 @@ def test_error_codes_on_gpu():
     with pytest.raises(psb.PSBError):
         psb.psb_build(np.full((10, 2), np.inf, np.float32), 32)
     idx.free()
+
+
+def test_host_buffers_and_stats(c2):
+    """Host (pinned and pageable) buffers through the C ABI give identical rows;
+    the instrumented entry point changes nothing and its counters are sane."""
+    psb = _psb()
+    cfg, pts, qs, idx, exp = c2
+    sl = slice(0, 2000)
+    e = (exp[0][sl], exp[1][sl])
+    hq = torch.from_numpy(qs[sl].copy()).pin_memory()
+    ids, d = psb.psb_knn(idx, hq, cfg.k)
+    torch.cuda.synchronize()
+    assert not ids.is_cuda
+    assert_same((ids.numpy(), d.numpy()), e, "pinned host buffers")
+    ids, d = psb.psb_knn(idx, torch.from_numpy(qs[sl].copy()), cfg.k,
+                         out=(torch.empty((2000, cfg.k), dtype=torch.int32),
+                              torch.empty((2000, cfg.k), dtype=torch.float32)))
+    torch.cuda.synchronize()
+    assert_same((ids.numpy(), d.numpy()), e, "pageable host buffers")
+    qd = torch.from_numpy(qs[sl].copy()).cuda()
+    for algo in (psb.PSB_ALGO_PSB, psb.PSB_ALGO_BNB):
+        got = []
+        for var in (0, 1):
+            i, dd, st = psb.psb_knn_stats(idx, qd, cfg.k, algo=algo, variant=var)
+            torch.cuda.synchronize()
+            assert_same((i.cpu().numpy(), dd.cpu().numpy()), e, f"stats algo={algo} var={var}")
+            st = st.cpu().numpy()
+            assert (st[:, 1] >= 1).all()                 # every query scans a leaf
+            assert (st[:, 0] >= idx.levels).all()        # and fetches at least one root-to-leaf path
+            got.append(st)
+        i2, _, st2 = psb.psb_knn_stats(idx, qd, cfg.k, algo=algo)
+        torch.cuda.synchronize()
+        assert np.array_equal(st2.cpu().numpy(), got[0])          # deterministic
+        assert (got[1][:, 3] == 0).all()                           # no cache -> no hits
+        assert np.array_equal(got[0][:, 0] + got[0][:, 3], got[1][:, 0])  # same visits, cache or not
+        assert np.array_equal(got[0][:, 1], got[1][:, 1])
