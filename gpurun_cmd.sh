@@ -1,4 +1,4 @@
-set -x
-timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -15
-timeout 600 python bench.py 2>&1 | tail -1 > gpurun_out/bench_c2.json; cat gpurun_out/bench_c2.json
-timeout 400 python tools/quick_time.py C1 C2 C3 2>&1 | tail -30
+timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
+for so in libpsb.so libpsb_mb8.so libpsb_mb10.so libpsb_mb12.so; do
+  echo "=== $so"; PSB_LIB_PATH=$PWD/paper_conf_icpp_namkn16_b200/$so timeout 300 python tools/quick_time.py C2 C3 2>&1 | grep -E "psb|bnb|C2|C3"
+done

@@ -19,7 +19,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libpsb.so")
+LIB_PATH = os.environ.get("PSB_LIB_PATH") or os.path.join(_HERE, "libpsb.so")   # override: A/B builds
 
 PSB_OK, PSB_EINVAL, PSB_ENOMEM, PSB_ECUDA, PSB_EUNSUPPORTED = 0, -1, -2, -3, -4
 PSB_PACK_HILBERT, PSB_PACK_STR = 0, 1

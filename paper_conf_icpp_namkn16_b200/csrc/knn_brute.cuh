@@ -56,11 +56,7 @@ brute_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k, 
             float p[V];
             ldv<V>(lp + j * F, p);
 #pragma unroll
-            for (int i = 0; i < QW; ++i) {
-                const float qj = q[i][j];
-#pragma unroll
-                for (int t = 0; t < V; ++t) dist[i][t] = __fadd_rn(dist[i][t], sq_diff(p[t], qj));
-            }
+            for (int i = 0; i < QW; ++i) acc_sq_diff<V>(dist[i], p, q[i][j]);
         });
         const int32_t *lid = ix.ids + leaf * F + lane * V;
 #pragma unroll

@@ -50,17 +50,17 @@ int launch_merge(const int32_t *ids, const float *dists, int parts, int64_t nq, 
 
 // Dispatch on d: specialised instantiations for the configs' d, runtime-d otherwise.
 int launch_tree(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                float *od, cudaStream_t st, uint32_t variant, int64_t *stats)
+                float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool)
 {
     int rc = PSB_NOT_INSTANTIATED;
     switch (ix.d) {
-    case 2: rc = launch_tree_v<2>(algo, ix, queries, nq, k, oi, od, st, variant, stats); break;
-    case 3: rc = launch_tree_v<3>(algo, ix, queries, nq, k, oi, od, st, variant, stats); break;
-    case 8: rc = launch_tree_v<8>(algo, ix, queries, nq, k, oi, od, st, variant, stats); break;
-    case 16: rc = launch_tree_v<16>(algo, ix, queries, nq, k, oi, od, st, variant, stats); break;
+    case 2: rc = launch_tree_v<2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool); break;
+    case 3: rc = launch_tree_v<3>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool); break;
+    case 8: rc = launch_tree_v<8>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool); break;
+    case 16: rc = launch_tree_v<16>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool); break;
     default: break;
     }
-    if (rc == PSB_NOT_INSTANTIATED) rc = launch_tree_v<0>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
+    if (rc == PSB_NOT_INSTANTIATED) rc = launch_tree_v<0>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
     return rc == PSB_NOT_INSTANTIATED ? PSB_EUNSUPPORTED : rc;
 }
 

@@ -13,6 +13,9 @@
 namespace psb {
 
 constexpr int WARPS_PER_CTA = 4;
+#ifndef PSB_MIN_BLOCKS
+#define PSB_MIN_BLOCKS 1
+#endif
 
 struct WarpState {
     float *cache_md;     // [(H+1)][F] child MINDISTs of the node cached per level
@@ -96,21 +99,21 @@ __device__ __forceinline__ int max_leaf(const DevIndex &ix, int lvl, int node)
     return (e < (int)ix.L ? e : (int)ix.L) - 1;
 }
 
+template <int F>
+struct Log2 {
+    static constexpr int value = F == 32 ? 5 : F == 64 ? 6 : F == 128 ? 7 : F == 256 ? 8 : 9;
+};
+
+// PSB for query qi, executed by one warp (Alg. 1 with the readings of DESIGN.md §2).
 template <int D, int V, int KS>
-__global__ void __launch_bounds__(WARPS_PER_CTA * 32)
-psb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
-           int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant,
-           int64_t *__restrict__ stats)
+__device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__restrict__ queries, int64_t qi,
+                                          int k, int32_t *__restrict__ out_ids, float *__restrict__ out_dists,
+                                          int64_t *__restrict__ stats, const WarpState &ws, bool use_cache,
+                                          bool use_max, int lane)
 {
     constexpr int F = 32 * V;
-    extern __shared__ __align__(16) unsigned char smem[];
-    const int lane = threadIdx.x & 31;
-    const int64_t qi = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
-    if (qi >= nq) return;
+    constexpr int LOGF = Log2<F>::value;
     const int H = ix.H;
-    const WarpState ws = warp_state(smem, H, F, D == 0);
-    const bool use_cache = !(variant & PSB_VAR_NOCACHE);
-    const bool use_max = !(variant & PSB_VAR_NOMAXDIST);
 
     // S1: query to registers, kNNs <- {inf} (Alg. 1 l.1-2)
     Query<D> q;
@@ -167,13 +170,18 @@ psb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
         if (lvl > 0) {
             float md[V];
             S.node(internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
-            // S6: eligible(c) = MINDIST <= pd (R5) and unvisited leaves below (R8)
-            const int base = node * F, nb = (int)ix.nlev[lvl - 1];
+            // S6: eligible(c) = MINDIST <= pd (R5) and unvisited leaves below (R8).
+            // Subtree leaf ranges are contiguous and increasing in c, so
+            // maxLeaf(child c) > visited  <=>  visited+1 < L  and
+            // base + c >= (visited+1) / F^(lvl-1)   (a warp-uniform threshold).
+            const int base = node * F;
+            const int c_end = min(F, (int)ix.nlev[lvl - 1] - base);
+            const int c_min = visited + 1 < (int)ix.L ? ((visited + 1) >> ((lvl - 1) * LOGF)) - base : F;
             unsigned mine = 0;
 #pragma unroll
             for (int t = 0; t < V; ++t) {
-                const int g = base + lane * V + t;
-                const bool e = g < nb && md[t] <= pd && max_leaf(ix, lvl - 1, g) > visited;
+                const int c = lane * V + t;
+                const bool e = c >= c_min && c < c_end && md[t] <= pd;
                 mine |= (unsigned)e << t;
             }
             const unsigned bal = __ballot_sync(FULL, mine != 0);
@@ -183,8 +191,8 @@ psb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
                 node = base + src * V + (__ffs(m) - 1);
                 --lvl;
             } else {                                             // S7 backtrack (R9)
+                if (lvl == H) break;                             // root exhausted (R10)
                 visited = max_leaf(ix, lvl, node);
-                if (lvl == H) break;
                 node /= F;
                 ++lvl;
             }
@@ -218,20 +226,13 @@ psb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
 // (MINDIST, index) order after the one we returned from, among those with
 // MINDIST <= pd; a leaf always returns to its parent.
 template <int D, int V, int KS>
-__global__ void __launch_bounds__(WARPS_PER_CTA * 32)
-bnb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
-           int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant,
-           int64_t *__restrict__ stats)
+__device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__restrict__ queries, int64_t qi,
+                                          int k, int32_t *__restrict__ out_ids, float *__restrict__ out_dists,
+                                          int64_t *__restrict__ stats, const WarpState &ws, bool use_cache,
+                                          bool use_max, int lane)
 {
     constexpr int F = 32 * V;
-    extern __shared__ __align__(16) unsigned char smem[];
-    const int lane = threadIdx.x & 31;
-    const int64_t qi = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
-    if (qi >= nq) return;
     const int H = ix.H;
-    const WarpState ws = warp_state(smem, H, F, D == 0);
-    const bool use_cache = !(variant & PSB_VAR_NOCACHE);
-    const bool use_max = !(variant & PSB_VAR_NOMAXDIST);
 
     Query<D> q;
     q.load(queries + qi * ix.d, ix.d, ws.qsmem);
@@ -291,43 +292,95 @@ bnb_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,
     S.write(stats, qi, lane);
 }
 
+
+// One warp per query. With `queue` non-null the grid is persistent (as many
+// CTAs as fit on the GPU) and each warp takes the next query from an atomic
+// counter when it finishes one, so a long query never holds an idle block.
+#define PSB_TREE_KERNEL(NAME, BODY)                                                                  \
+    template <int D, int V, int KS>                                                                   \
+    __global__ void __launch_bounds__(WARPS_PER_CTA * 32, PSB_MIN_BLOCKS)                            \
+    NAME(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,                          \
+         int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant,             \
+         int64_t *__restrict__ stats, unsigned long long *__restrict__ queue)                        \
+    {                                                                                                 \
+        extern __shared__ __align__(16) unsigned char smem[];                                         \
+        const int lane = threadIdx.x & 31;                                                            \
+        const WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0);                                  \
+        const bool use_cache = !(variant & PSB_VAR_NOCACHE);                                          \
+        const bool use_max = !(variant & PSB_VAR_NOMAXDIST);                                          \
+        int64_t qi = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);                        \
+        while (true) {                                                                                \
+            if (queue) {                                                                              \
+                unsigned long long v = 0;                                                             \
+                if (lane == 0) v = atomicAdd(queue, 1ull);                                            \
+                qi = (int64_t)__shfl_sync(FULL, v, 0);                                                \
+            }                                                                                         \
+            if (qi >= nq) break;                                                                      \
+            BODY<D, V, KS>(ix, queries, qi, k, out_ids, out_dists, stats, ws, use_cache, use_max, lane); \
+            if (!queue) break;                                                                        \
+        }                                                                                             \
+    }
+
+PSB_TREE_KERNEL(psb_kernel, psb_query)
+PSB_TREE_KERNEL(bnb_kernel, bnb_query)
+
 template <int D, int V, int KS>
 static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
-                         int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats)
+                         int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats,
+                         cudaMemPool_t pool)
 {
     const size_t smem = WARPS_PER_CTA * WarpSmem::bytes(ix.H, 32 * V, D == 0);
-    const int64_t blocks = (nq + WARPS_PER_CTA - 1) / WARPS_PER_CTA;
+    int64_t blocks = (nq + WARPS_PER_CTA - 1) / WARPS_PER_CTA;
     auto kern = algo == PSB_ALGO_PSB ? psb_kernel<D, V, KS> : bnb_kernel<D, V, KS>;
+    cudaError_t e;
     if (smem > 48 * 1024) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return report_cuda(e, "cudaFuncSetAttribute");
     }
-    kern<<<(unsigned)blocks, WARPS_PER_CTA * 32, smem, st>>>(ix, queries, nq, k, oi, od, variant, stats);
-    return report_cuda(cudaGetLastError(), "tree kernel launch");
+    // More queries than resident warps: persistent grid + atomic query queue.
+    int per_sm = 0;
+    unsigned long long *queue = nullptr;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, WARPS_PER_CTA * 32, smem) == cudaSuccess &&
+        per_sm > 0 && blocks > (int64_t)per_sm * ix.sm_count) {
+        if ((e = cudaMallocFromPoolAsync((void **)&queue, sizeof(unsigned long long), pool, st)) != cudaSuccess)
+            return report_cuda(e, "cudaMallocFromPoolAsync (query queue)");
+        if ((e = cudaMemsetAsync(queue, 0, sizeof(unsigned long long), st)) != cudaSuccess) {
+            cudaFreeAsync(queue, st);
+            return report_cuda(e, "cudaMemsetAsync (query queue)");
+        }
+        blocks = (int64_t)per_sm * ix.sm_count;
+    }
+    cudaGetLastError();
+    kern<<<(unsigned)blocks, WARPS_PER_CTA * 32, smem, st>>>(ix, queries, nq, k, oi, od, variant, stats, queue);
+    int rc = report_cuda(cudaGetLastError(), "tree kernel launch");
+    if (queue) cudaFreeAsync(queue, st);
+    return rc;
 }
 
 template <int D, int V>
 static int launch_tree_ks(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
-                          int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats)
+                          int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats,
+                         cudaMemPool_t pool)
 {
-    if (k <= 32) return launch_tree_t<D, V, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
-    if (k <= 64) return launch_tree_t<D, V, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
-    return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
+    if (k <= 32) return launch_tree_t<D, V, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
+    if (k <= 64) return launch_tree_t<D, V, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
+    return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
 }
 
 template <int D>
 int launch_tree_v(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
-                         int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats)
+                         int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats,
+                         cudaMemPool_t pool)
 {
     switch (ix.F) {
-    case 32: return launch_tree_ks<D, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
-    case 64: return launch_tree_ks<D, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
-    case 128: return launch_tree_ks<D, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
+    case 32: return launch_tree_ks<D, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
+    case 64: return launch_tree_ks<D, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
+    case 128: return launch_tree_ks<D, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
     default: break;
     }
     if constexpr (D == 0) {
-        if (ix.F == 256) return launch_tree_ks<0, 8>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
-        if (ix.F == 512) return launch_tree_ks<0, 16>(algo, ix, queries, nq, k, oi, od, st, variant, stats);
+        if (ix.F == 256) return launch_tree_ks<0, 8>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
+        if (ix.F == 512) return launch_tree_ks<0, 16>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
     }
     return PSB_NOT_INSTANTIATED;   // caller falls back to the generic-d kernels
 }

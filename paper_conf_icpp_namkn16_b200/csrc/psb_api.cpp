@@ -85,6 +85,7 @@ static DevIndex dev_view(const psb_index *ix)
     v.H = ix->H;
     v.d = ix->d;
     v.F = ix->F;
+    v.sm_count = ix->sm_count;
     return v;
 }
 
@@ -254,7 +255,7 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
     if (rc == PSB_OK) {
         const DevIndex v = dev_view(ix);
         rc = algo == PSB_ALGO_BRUTE ? psb::launch_brute(v, dq, q, k, di, dd, st, ix->sm_count, ix->pool)
-                                    : psb::launch_tree(algo, v, dq, q, k, di, dd, st, variant, stats);
+                                    : psb::launch_tree(algo, v, dq, q, k, di, dd, st, variant, stats, ix->pool);
     }
     if (ho) {
         if (rc == PSB_OK && ((e = cudaMemcpyAsync(out_ids, di, bo, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||

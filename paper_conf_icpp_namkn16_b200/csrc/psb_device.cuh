@@ -39,6 +39,53 @@ __device__ __forceinline__ float sq_diff(float a, float b)
     return __fmul_rn(t, t);
 }
 
+// Packed binary32 pairs (sm_100 FADD2 / FMUL2): each half is rounded exactly as
+// the scalar op. ptxas 12.9 contracts a mul.rn.f32x2 that feeds an
+// add.rn.f32x2 into FFMA2 even with --fmad=false, which would break the RN
+// contract; so only the difference and the square are packed and the running
+// sums stay scalar __fadd_rn (tests/test_abi_host.py checks the SASS has no FFMA).
+__device__ __forceinline__ u64 f2_pack(float a, float b)
+{
+    u64 r;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(a), "f"(b));
+    return r;
+}
+__device__ __forceinline__ void f2_unpack(u64 r, float &a, float &b)
+{
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(r));
+}
+__device__ __forceinline__ u64 f2_sub(u64 a, u64 b)
+{
+    u64 r;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ u64 f2_mul(u64 a, u64 b)
+{
+    u64 r;
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+// dist[t] += (p[t] - q)^2 for V points, pairs packed when V is even.
+template <int V>
+__device__ __forceinline__ void acc_sq_diff(float (&dist)[V], const float (&p)[V], float qj)
+{
+    if constexpr (V % 2 == 0) {
+        const u64 qq = f2_pack(qj, qj);
+#pragma unroll
+        for (int t = 0; t < V; t += 2) {
+            const u64 d2 = f2_sub(f2_pack(p[t], p[t + 1]), qq);
+            float a, b;
+            f2_unpack(f2_mul(d2, d2), a, b);
+            dist[t] = __fadd_rn(dist[t], a);
+            dist[t + 1] = __fadd_rn(dist[t + 1], b);
+        }
+    } else {
+#pragma unroll
+        for (int t = 0; t < V; ++t) dist[t] = __fadd_rn(dist[t], sq_diff(p[t], qj));
+    }
+}
+
 // Loop over dimensions 0..d-1 in order: fully unrolled for a compile-time D (so
 // query coordinates stay in registers), a runtime loop otherwise.
 template <int D, typename Body>
@@ -135,9 +182,7 @@ __device__ __forceinline__ void leaf_dists(const float *__restrict__ lp, const Q
     for_dims<D>(d, [&](int j) {
         float p[V];
         ldv<V>(lp + j * F + lane * V, p);
-        const float qj = q[j];
-#pragma unroll
-        for (int t = 0; t < V; ++t) dist[t] = __fadd_rn(dist[t], sq_diff(p[t], qj));
+        acc_sq_diff<V>(dist, p, q[j]);
     });
 }
 
@@ -183,10 +228,14 @@ __device__ __forceinline__ u64 cmpx(u64 v, int j, bool take_min)
     const u64 o = __shfl_xor_sync(FULL, v, j);
     return take_min ? (o < v ? o : v) : (o < v ? v : o);
 }
+// Sorts each group of G lanes (G = 8, 16 or 32; groups alternate direction).
+// With candidates in lanes 0..G-1 and ~0 everywhere else, the whole warp is
+// then ascending.
+template <int G = 32>
 __device__ __forceinline__ u64 warp_sort32(u64 v, int lane)
 {
 #pragma unroll
-    for (int kk = 2; kk <= 32; kk <<= 1) {
+    for (int kk = 2; kk <= G; kk <<= 1) {
         const bool asc = (lane & kk) == 0;
 #pragma unroll
         for (int j = kk >> 1; j > 0; j >>= 1) v = cmpx(v, j, ((lane & j) == 0) == asc);
@@ -247,9 +296,10 @@ struct TopK {
     // the elementwise min/max against the reversed candidates (the 32 smallest /
     // largest of the union, each a bitonic sequence) and re-sort both halves;
     // the larger half carries into the next segment, the last one is dropped.
+    template <int G = 32>
     __device__ __forceinline__ void merge32(u64 c, int lane)
     {
-        c = warp_sort32(c, lane);
+        c = warp_sort32<G>(c, lane);
 #pragma unroll
         for (int s = 0; s < KS; ++s) {
             const u64 rc = __shfl_sync(FULL, c, 31 - lane);
@@ -301,7 +351,9 @@ struct TopK {
             __syncwarp();
             const u64 c = lane < m ? scratch[lane] : ~0ull;
             __syncwarp();
-            merge32(c, lane);
+            if (m <= 8) merge32<8>(c, lane);
+            else if (m <= 16) merge32<16>(c, lane);
+            else merge32<32>(c, lane);
         } else {
 #pragma unroll
             for (int t = 0; t < V; ++t) {

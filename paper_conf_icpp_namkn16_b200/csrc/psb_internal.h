@@ -27,6 +27,7 @@ struct DevIndex {
     int32_t H;                          // internal levels; root = (H, 0)
     int32_t d;
     int32_t F;
+    int32_t sm_count;                   // of the index's device (launch sizing)
 };
 
 struct HostLayout {

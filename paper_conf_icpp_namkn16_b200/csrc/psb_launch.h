@@ -13,7 +13,7 @@ int report_cuda(cudaError_t e, const char *what);
 // `stats` (nullable, device [nq][4] int64): per query {internal node fetches,
 // leaf scans, id loads, path-cache hits}.
 int launch_tree(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                float *od, cudaStream_t st, uint32_t variant, int64_t *stats);
+                float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool);
 
 // Exhaustive scan of all points (knn_brute.cu). Splits the point set into
 // chunks when there are too few queries to fill the GPU and merges the partial
@@ -26,7 +26,7 @@ int launch_brute(const DevIndex &ix, const float *queries, int64_t nq, int k, in
 constexpr int PSB_NOT_INSTANTIATED = 1;
 template <int D>
 int launch_tree_v(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                  float *od, cudaStream_t st, uint32_t variant, int64_t *stats);
+                  float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool);
 template <int D>
 int launch_brute_v(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi, float *od,
                    cudaStream_t st, int sm, cudaMemPool_t pool);

@@ -164,3 +164,16 @@ def test_pack_modes_and_id_base_only_change_layout():
     assert np.array_equal(a["ids"][a["ids"] >= 0] + 1000, b["ids"][b["ids"] >= 0])
     s = psb.psb_build_host_blob(pts, 32, packing=psb.PSB_PACK_STR)
     assert sorted(s["ids"][s["ids"] >= 0].tolist()) == list(range(3000))
+
+
+def test_sass_has_no_fused_multiply_add():
+    """Bit-exactness guard: no FFMA/FFMA2 anywhere in libpsb.so's sm_100a SASS
+    (the distance and the bounds are sub, mul, add each rounded once, R14).
+    ptxas contracts mul.f32x2 -> add.f32x2 into FFMA2 even with --fmad=false,
+    so this check is what keeps the packed FADD2/FMUL2 path honest."""
+    import subprocess
+    sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", psb.LIB_PATH],
+                          capture_output=True, text=True).stdout
+    assert "FADD" in sass and "FMUL" in sass
+    fused = [l for l in sass.splitlines() if re.search(r"\bFFMA2?\b|\bDFMA\b", l)]
+    assert not fused, fused[:5]
