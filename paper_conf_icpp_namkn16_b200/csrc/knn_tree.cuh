@@ -14,7 +14,7 @@ namespace psb {
 
 constexpr int WARPS_PER_CTA = 4;
 #ifndef PSB_MIN_BLOCKS
-#define PSB_MIN_BLOCKS 1
+#define PSB_MIN_BLOCKS 8   // <= 64 registers: measured best on C2/C3 (profiles/r01_occupancy.md)
 #endif
 
 struct WarpState {
