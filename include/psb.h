@@ -121,9 +121,10 @@ int psb_knn_ex(const psb_index *idx, const float *queries, int64_t q, int32_t k,
 enum { PSB_ALGO_PSB = 0, PSB_ALGO_BNB = 1, PSB_ALGO_BRUTE = 2 };
 
 /* psb_knn_ex (algo PSB_ALGO_PSB or PSB_ALGO_BNB) that also writes per-query
- * traversal counters to `stats`, a DEVICE array int64[q][4]:
+ * traversal counters to `stats`, a DEVICE array int64[q][8]:
  *   {internal-node fetches from memory, leaf scans, point ids loaded,
- *    internal-node visits served by the path cache}.
+ *    internal-node visits served by the path cache, leaf scans that changed the
+ *    kNN list, keys merged into the list, 0, 0}.
  * The counters define the algorithmic bytes of a launch:
  *   fetches*fanout*2*d*4 + leaf_scans*fanout*d*4 + ids*4 + q*(4*d + 8*k).
  * The traversal (and hence every counter) is deterministic: a counting run and

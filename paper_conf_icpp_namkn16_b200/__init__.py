@@ -182,11 +182,12 @@ def psb_knn_ex(index: Index, queries, k: int, algo: int = PSB_ALGO_PSB, variant:
 
 def psb_knn_stats(index: Index, queries, k: int, algo: int = PSB_ALGO_PSB, variant: int = 0,
                   stream=None, out=None):
-    """psb_knn_ex plus per-query counters: returns (ids, dists, stats int64 [q, 4] on device)
-    with stats = {node fetches, leaf scans, id loads, path-cache hits}."""
+    """psb_knn_ex plus per-query counters: returns (ids, dists, stats int64 [q, 8] on device)
+    with stats = {node fetches, leaf scans, id loads, path-cache hits, changing leaf scans,
+    keys merged, 0, 0} (include/psb.h)."""
     torch = _torch()
     queries, q, ids, dists = _query_buffers(index, queries, k, out)
-    stats = torch.zeros((q, 4), dtype=torch.int64, device=f"cuda:{index.device}")
+    stats = torch.zeros((q, 8), dtype=torch.int64, device=f"cuda:{index.device}")
     _check(_lib.psb_knn_stats(index.handle, queries.data_ptr(), q, k, ids.data_ptr(), dists.data_ptr(),
                               _stream_handle(stream), algo, variant, stats.data_ptr()), "psb_knn_stats")
     return ids, dists, stats

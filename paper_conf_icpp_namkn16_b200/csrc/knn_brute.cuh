@@ -121,7 +121,8 @@ static int launch_brute_ks(const DevIndex &ix, const float *queries, int64_t nq,
 {
     if (k <= 32) return launch_brute_t<D, V, 1>(ix, queries, nq, k, oi, od, st, sm, pool);
     if (k <= 64) return launch_brute_t<D, V, 2>(ix, queries, nq, k, oi, od, st, sm, pool);
-    return launch_brute_t<D, V, 4>(ix, queries, nq, k, oi, od, st, sm, pool);
+    if constexpr (D == 0) return launch_brute_t<D, V, 4>(ix, queries, nq, k, oi, od, st, sm, pool);
+    return PSB_NOT_INSTANTIATED;   // k > 64: generic-d kernels
 }
 
 template <int D>

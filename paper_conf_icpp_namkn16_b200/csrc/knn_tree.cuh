@@ -75,22 +75,6 @@ __device__ __forceinline__ bool internal_md(const DevIndex &ix, int lvl, int nod
     return true;
 }
 
-// Per-query traversal counters (psb_knn_stats): they define the algorithmic
-// bytes of SURVEY.md §8(d) without changing the traversal.
-struct Stats {
-    uint32_t fetch = 0, hit = 0, leaf = 0, ids = 0;
-    __device__ __forceinline__ void node(bool fetched) { fetched ? ++fetch : ++hit; }
-    __device__ __forceinline__ void write(int64_t *st, int64_t qi, int lane) const
-    {
-        if (st && lane == 0) {
-            st[qi * 4 + 0] = fetch;
-            st[qi * 4 + 1] = leaf;
-            st[qi * 4 + 2] = ids;
-            st[qi * 4 + 3] = hit;
-        }
-    }
-};
-
 // Last leaf under (lvl, node): min((node+1)*F^lvl, L) - 1. With span clamped at
 // L and node < F*nlev[lvl], the product stays below 2L < 2^27 (n < 2^31, F >= 32).
 __device__ __forceinline__ int max_leaf(const DevIndex &ix, int lvl, int node)
@@ -105,7 +89,7 @@ struct Log2 {
 };
 
 // PSB for query qi, executed by one warp (Alg. 1 with the readings of DESIGN.md §2).
-template <int D, int V, int KS>
+template <int D, int V, int KS, bool ST>
 __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__restrict__ queries, int64_t qi,
                                           int k, int32_t *__restrict__ out_ids, float *__restrict__ out_dists,
                                           int64_t *__restrict__ stats, const WarpState &ws, bool use_cache,
@@ -124,7 +108,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     T.init();
     u64 thr = PAD_KEY;
     float pd = __int_as_float(0x7f800000);
-    Stats S;
+    Stats<ST> S;
 
     // S2: pass 1, getInitialPruningDistance(Q, ClosestLeaf) (Alg. 1 l.3; R4):
     // greedy descent by (MINDIST, child index) argmin, k-th-MAXDIST bounds on the way.
@@ -154,8 +138,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     int64_t seen = 0;
     while (seen < k && pass1_hi + 1 < (int)ix.L) {
         ++pass1_hi;
-        scan_leaf<D, V, KS>(ix, pass1_hi, q, lane, T, k, thr, S.ids, ws.scratch);
-        ++S.leaf;
+        scan_leaf<D, V, KS, ST>(ix, pass1_hi, q, lane, T, k, thr, S, ws.scratch);
         const int64_t left = ix.n - (int64_t)pass1_hi * F;
         seen += left < F ? left : F;
     }
@@ -203,8 +186,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
             if (j >= pass1_lo && j <= pass1_hi) {
                 changed = true;                                  // already offered in pass 1
             } else {
-                changed = scan_leaf<D, V, KS>(ix, j, q, lane, T, k, thr, S.ids, ws.scratch);
-                ++S.leaf;
+                changed = scan_leaf<D, V, KS, ST>(ix, j, q, lane, T, k, thr, S, ws.scratch);
             }
             pd = fminf(pd, key_dist(thr));                       // Alg. 1 l.37
             visited = j;                                         // l.38
@@ -225,7 +207,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
 // Stackless B&B: at an internal node take the next child in
 // (MINDIST, index) order after the one we returned from, among those with
 // MINDIST <= pd; a leaf always returns to its parent.
-template <int D, int V, int KS>
+template <int D, int V, int KS, bool ST>
 __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__restrict__ queries, int64_t qi,
                                           int k, int32_t *__restrict__ out_ids, float *__restrict__ out_dists,
                                           int64_t *__restrict__ stats, const WarpState &ws, bool use_cache,
@@ -242,7 +224,7 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
     T.init();
     u64 thr = PAD_KEY;
     float pd = __int_as_float(0x7f800000);
-    Stats S;
+    Stats<ST> S;
 
     int lvl = H;
     int node = 0;
@@ -280,8 +262,7 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
                 ++lvl;
             }
         } else {
-            scan_leaf<D, V, KS>(ix, node, q, lane, T, k, thr, S.ids, ws.scratch);
-            ++S.leaf;
+            scan_leaf<D, V, KS, ST>(ix, node, q, lane, T, k, thr, S, ws.scratch);
             pd = fminf(pd, key_dist(thr));
             from_c = (int)(node % F);
             node /= F;
@@ -297,7 +278,7 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
 // CTAs as fit on the GPU) and each warp takes the next query from an atomic
 // counter when it finishes one, so a long query never holds an idle block.
 #define PSB_TREE_KERNEL(NAME, BODY)                                                                  \
-    template <int D, int V, int KS>                                                                   \
+    template <int D, int V, int KS, bool ST>                                                          \
     __global__ void __launch_bounds__(WARPS_PER_CTA * 32, PSB_MIN_BLOCKS)                            \
     NAME(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,                          \
          int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant,             \
@@ -316,7 +297,7 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
                 qi = (int64_t)__shfl_sync(FULL, v, 0);                                                \
             }                                                                                         \
             if (qi >= nq) break;                                                                      \
-            BODY<D, V, KS>(ix, queries, qi, k, out_ids, out_dists, stats, ws, use_cache, use_max, lane); \
+            BODY<D, V, KS, ST>(ix, queries, qi, k, out_ids, out_dists, stats, ws, use_cache, use_max, lane); \
             if (!queue) break;                                                                        \
         }                                                                                             \
     }
@@ -331,7 +312,8 @@ static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int
 {
     const size_t smem = WARPS_PER_CTA * WarpSmem::bytes(ix.H, 32 * V, D == 0);
     int64_t blocks = (nq + WARPS_PER_CTA - 1) / WARPS_PER_CTA;
-    auto kern = algo == PSB_ALGO_PSB ? psb_kernel<D, V, KS> : bnb_kernel<D, V, KS>;
+    auto kern = algo == PSB_ALGO_PSB ? (stats ? psb_kernel<D, V, KS, true> : psb_kernel<D, V, KS, false>)
+                                     : (stats ? bnb_kernel<D, V, KS, true> : bnb_kernel<D, V, KS, false>);
     cudaError_t e;
     if (smem > 48 * 1024) {
         e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -364,7 +346,8 @@ static int launch_tree_ks(int algo, const DevIndex &ix, const float *queries, in
 {
     if (k <= 32) return launch_tree_t<D, V, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
     if (k <= 64) return launch_tree_t<D, V, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
-    return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
+    if constexpr (D == 0) return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
+    return PSB_NOT_INSTANTIATED;   // k > 64: generic-d kernels (keeps compile time down)
 }
 
 template <int D>

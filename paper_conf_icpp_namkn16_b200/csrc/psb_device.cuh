@@ -309,12 +309,12 @@ struct TopK {
             if (s + 1 < KS) c = warp_merge32(hi, lane);
         }
     }
-    // Offer this lane's V candidate keys (~0 = none); returns whether any entered
-    // the first k positions. `thr` is the k-th key, kept current. Few candidates
+    // Offer this lane's V candidate keys (~0 = none); returns how many were below
+    // the k-th key (> 0 iff the first k positions changed). `thr` is the k-th key, kept current. Few candidates
     // are inserted one by one; more are compacted through `scratch` (32 u64 of
     // per-warp shared memory) and merged 32 at a time.
     template <int V>
-    __device__ __forceinline__ bool offer(const u64 (&cand)[V], int k, int lane, u64 &thr, u64 *scratch)
+    __device__ __forceinline__ int offer(const u64 (&cand)[V], int k, int lane, u64 &thr, u64 *scratch)
     {
         unsigned bal[V];
         int m = 0;
@@ -323,7 +323,7 @@ struct TopK {
             bal[t] = __ballot_sync(FULL, cand[t] < thr);
             m += __popc(bal[t]);
         }
-        if (m == 0) return false;
+        if (m == 0) return 0;
         if (m <= 2) {
 #pragma unroll
             for (int t = 0; t < V; ++t) {
@@ -338,7 +338,7 @@ struct TopK {
                     }
                 }
             }
-            return true;
+            return m;
         }
         if (m <= 32) {
             const unsigned lt = (1u << lane) - 1;
@@ -365,7 +365,7 @@ struct TopK {
             }
         }
         thr = kth(k);
-        return true;
+        return m;
     }
     __device__ __forceinline__ void store(int k, int lane, int32_t *__restrict__ oi,
                                           float *__restrict__ od) const
@@ -381,15 +381,43 @@ struct TopK {
     }
 };
 
+// Per-query traversal counters (psb_knn_stats, int64[q][8]). They define the
+// algorithmic bytes of a launch without changing the traversal.
+// Compiled in only for the psb_knn_stats instantiations (ON = true): the timed
+// kernels carry no counting code.
+template <bool ON>
+struct Stats {
+    uint32_t fetch = 0, hit = 0, leaf = 0, ids = 0, offers = 0, cand = 0;
+    __device__ __forceinline__ void node(bool fetched) { if (ON) { fetched ? ++fetch : ++hit; } }
+    __device__ __forceinline__ void scan() { if (ON) ++leaf; }
+    __device__ __forceinline__ void id_loads(int n) { if (ON) ids += n; }
+    __device__ __forceinline__ void merged(int m) { if (ON) { cand += m; offers += m > 0; } }
+    __device__ __forceinline__ void write(int64_t *st, int64_t qi, int lane) const
+    {
+        if (ON && lane == 0) {
+            int64_t *o = st + qi * 8;
+            o[0] = fetch;   // internal-node blocks fetched from memory
+            o[1] = leaf;    // leaf blocks scanned
+            o[2] = ids;     // point ids loaded
+            o[3] = hit;     // internal visits served by the path cache
+            o[4] = offers;  // leaf scans that changed the kNN list
+            o[5] = cand;    // keys merged into the kNN list
+            o[6] = 0;
+            o[7] = 0;
+        }
+    }
+};
+
 // S8+S9: scan one leaf, offer its points. Ids are fetched lazily, only for
 // points whose distance can enter the list (dist <= current k-th distance).
-template <int D, int V, int KS>
+template <int D, int V, int KS, bool ST>
 __device__ __forceinline__ bool scan_leaf(const DevIndex &ix, int leaf, const Query<D> &q,
-                                          int lane, TopK<KS> &T, int k, u64 &thr, uint32_t &n_ids,
+                                          int lane, TopK<KS> &T, int k, u64 &thr, Stats<ST> &S,
                                           u64 *scratch)
 {
     constexpr int F = 32 * V;
     float dist[V];
+    S.scan();
     leaf_dists<D, V>(ix.pts + (int64_t)leaf * ix.d * F, q, ix.d, lane, dist);
     const float td = key_dist(thr);
     bool any = false;
@@ -404,8 +432,10 @@ __device__ __forceinline__ bool scan_leaf(const DevIndex &ix, int leaf, const Qu
         cand[t] = dist[t] <= td ? make_key(dist[t], __ldg(lid + t)) : ~0ull;
         loads += dist[t] <= td;
     }
-    n_ids += __reduce_add_sync(FULL, loads);
-    return T.template offer<V>(cand, k, lane, thr, scratch);
+    if (ST) S.id_loads(__reduce_add_sync(FULL, loads));
+    const int m = T.template offer<V>(cand, k, lane, thr, scratch);
+    S.merged(m);
+    return m > 0;
 }
 
 // Per-warp shared-memory layout for the traversal kernels.

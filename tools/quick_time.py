@@ -5,7 +5,7 @@ import numpy as np, torch
 import paper_conf_icpp_namkn16_b200 as psb
 import workloads as W
 
-def time_it(fn, reps=5):
+def time_it(fn, reps=15):
     s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     fn(); torch.cuda.synchronize()
     ts = []
@@ -23,6 +23,6 @@ for name in sys.argv[1:] or ["C1", "C2", "C3"]:
         for var in ((0, 1) if an < 2 else (0,)):
             if an == 2 and cfg.n * cfg.q > 2e10: 
                 continue
-            mn, med = time_it(lambda: psb.psb_knn_ex(idx, qd, cfg.k, algo=an, variant=var), 3)
-            print(f"  {algo:6s} var{var}: {med:9.3f} ms  {cfg.q/med*1e3/1e6:8.3f} Mq/s", flush=True)
+            mn, med = time_it(lambda: psb.psb_knn_ex(idx, qd, cfg.k, algo=an, variant=var))
+            print(f"  {algo:6s} var{var}: {med:9.3f} ms (min {mn:.3f})  {cfg.q/med*1e3/1e6:8.3f} Mq/s", flush=True)
     idx.free()
