@@ -362,8 +362,7 @@ def main():
                                                 {"node_fetches": stats_sum[0] / q, "leaf_scans": stats_sum[1] / q,
                                                  "id_loads": stats_sum[2] / q, "cache_hits": stats_sum[3] / q,
                                                  "changing_leaf_scans": stats_sum[4] / q,
-                                                 "keys_merged": stats_sum[5] / q,
-                                                 "leaves_skipped": stats_sum[6] / q})},
+                                                 "keys_merged": stats_sum[5] / q})},
             "clocks": clocks,
             "gpu_launches": args.steps * (1 if args.algo != "brute" else 2) * (1 if args.mode == "query" or world == 1 else 2),
             **extras,
