@@ -47,6 +47,8 @@ def parse():
     ap.add_argument("--config", default="C2", choices=sorted(W.CONFIGS))
     ap.add_argument("--queries", type=int, default=0, help="override q per step (0 = config's)")
     ap.add_argument("--mode", default="query", choices=["query", "data"])
+    ap.add_argument("--slab", type=int, default=0,
+                    help="data mode on ONE GPU: run rank 0's local step of a P-way data-sharded job")
     ap.add_argument("--algo", default="psb", choices=["psb", "bnb", "brute"])
     ap.add_argument("--variant", type=int, default=0)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -212,15 +214,19 @@ def main():
     q = args.queries or cfg.q
     k = cfg.k
     algo = {"psb": psb.PSB_ALGO_PSB, "bnb": psb.PSB_ALGO_BNB, "brute": psb.PSB_ALGO_BRUTE}[args.algo]
-    pts = cfg.points()
     if args.mode == "query":
         # weak scaling: rank r answers its own batch of q queries on a replica
+        pts = cfg.points()
         all_q = cfg.queries(q * world)
         qs = all_q[rank * q:(rank + 1) * q]
         idx = psb.psb_build(pts, cfg.fanout)
     else:
+        # rank r holds slab r of the points (global ids via id_base); all ranks see all q queries
+        parts = max(world, args.slab or 1)
+        b = pdist.shard_bounds(cfg.n, parts)
+        pts = cfg.points(n=b[rank + 1] - b[rank], row0=b[rank])
         qs = cfg.queries(q)
-        idx = pdist.build_shard(pts, cfg.fanout, world, rank)
+        idx = psb.psb_build_ex(pts, cfg.fanout, id_base=b[rank])
     stream = torch.cuda.current_stream()
     qd = torch.from_numpy(qs).cuda()
     out_i = torch.empty((q, k), dtype=torch.int32, device="cuda")
@@ -323,7 +329,11 @@ def main():
         # comparators on the same batch (same timing protocol, fewer steps)
         comp = {}
         for name, a in (("psb", psb.PSB_ALGO_PSB), ("bnb", psb.PSB_ALGO_BNB), ("brute", psb.PSB_ALGO_BRUTE)):
-            reps = 20 if name != "brute" else 5
+            if name == "brute" and idx.n * q > 2e11:
+                comp[name] = {"skipped": f"n*q = {idx.n * q:.2e} pairs (minutes per batch)"}
+                continue
+            reps = 20 if name != "brute" else 3
+            reps = reps if q * idx.n < 1e12 else 3
             ts = []
             for i in range(reps + 2):
                 flush.fill_(i & 0xFF)
@@ -338,7 +348,7 @@ def main():
         extras["comparators_1gpu"] = comp
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and (args.mode == "query" or (args.slab or 1) == 1):
         psb.psb_knn_ex(idx, qd, k, algo=algo, variant=args.variant, out=(out_i, out_d))
         torch.cuda.synchronize()
         cpu = cpu_baseline(cfg, pts, qs, k, out_i.cpu().numpy(), out_d.cpu().numpy())
@@ -352,7 +362,9 @@ def main():
             "data": "synthetic (workloads/: seeded SplitMix64 uniform / 100-cluster Gaussian)",
             "config": {**cfg.describe(), "q": q, "algo": args.algo, "variant": args.variant,
                        "parallelism": (f"query-sharded x{world} (replicated index)" if args.mode == "query"
-                                       else f"data-sharded x{world} (NCCL all-gather + merge)"),
+                                       else (f"data-sharded x{world} (NCCL all-gather + merge)" if world > 1 else
+                                             f"data-sharded slab 0 of {max(1, args.slab)} (local step only, 1 GPU)")),
+                       "points_on_this_gpu": int(pts.shape[0]),
                        "l2": "flushed between steps (256 MiB write)", "index_bytes": idx.device_bytes},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "kernel": kernel,

@@ -57,6 +57,11 @@ enum {
 /* Leaf packing order for psb_build_ex `flags` (§IV-A: sort points by
  * a space-filling-curve key and pack them into full leaves, bottom-up). */
 enum { PSB_PACK_HILBERT = 0, PSB_PACK_STR = 1 };
+/* Build-location flag (OR into psb_build_ex `flags`). Hilbert packing runs on
+ * the GPU by default (keys, CUB radix sort, permutation and MBR levels in CUDA
+ * kernels; NEXT-1); PSB_BUILD_HOST forces the host (OpenMP) loader. STR always
+ * runs on the host. Both loaders produce the same index. */
+#define PSB_BUILD_HOST 0x100u
 
 #define PSB_KMAX 128          /* largest k served by the warp top-k (4 keys per lane) */
 #define PSB_DMAX 64           /* largest dimensionality                               */
@@ -80,7 +85,8 @@ psb_index *psb_build(const float *points, int64_t n, int32_t d, int32_t fanout);
 /* As psb_build, plus: returned ids are id_base + input row (data-sharded use:
  * a shard over rows [r0, r1) of a global set passes id_base = r0;
  * id_base >= 0 and id_base + n <= 2^31 - 1), and `flags` selects the packing
- * (PSB_PACK_HILBERT or PSB_PACK_STR). On success *out receives the index. */
+ * (PSB_PACK_HILBERT or PSB_PACK_STR, optionally | PSB_BUILD_HOST). On success
+ * *out receives the index. */
 int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int64_t id_base,
                  uint32_t flags, psb_index **out);
 

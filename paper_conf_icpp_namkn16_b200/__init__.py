@@ -23,6 +23,7 @@ LIB_PATH = os.environ.get("PSB_LIB_PATH") or os.path.join(_HERE, "libpsb.so")   
 
 PSB_OK, PSB_EINVAL, PSB_ENOMEM, PSB_ECUDA, PSB_EUNSUPPORTED = 0, -1, -2, -3, -4
 PSB_PACK_HILBERT, PSB_PACK_STR = 0, 1
+PSB_BUILD_HOST = 0x100
 PSB_ALGO_PSB, PSB_ALGO_BNB, PSB_ALGO_BRUTE = 0, 1, 2
 PSB_VAR_NOCACHE, PSB_VAR_NOMAXDIST = 1, 2
 PSB_KMAX, PSB_DMAX = 128, 64

@@ -109,47 +109,87 @@ int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int6
     int dev = -1;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return report_cuda(e, "psb_build_ex: cudaGetDevice");
-    // points may be host or device memory; the bulk load runs on the host
+    GpuLayoutShape shape;
+    int rc = psb_layout_shape(n, d, fanout, id_base, flags, &shape);
+    if (rc != PSB_OK) return rc;
+    const bool on_gpu = (flags & ~(uint32_t)PSB_BUILD_HOST) == PSB_PACK_HILBERT && !(flags & PSB_BUILD_HOST);
     cudaPointerAttributes attr;
-    const float *host_pts = points;
-    float *staged = nullptr;
     e = cudaPointerGetAttributes(&attr, points);
     if (e != cudaSuccess) {
         cudaGetLastError();
         attr.type = cudaMemoryTypeUnregistered;
     }
-    if (attr.type == cudaMemoryTypeDevice) {
-        staged = (float *)malloc(sizeof(float) * (size_t)(n * d));
-        if (!staged) { psb_set_error("psb_build_ex: host staging allocation failed"); return PSB_ENOMEM; }
-        e = cudaMemcpy(staged, points, sizeof(float) * (size_t)(n * d), cudaMemcpyDeviceToHost);
-        if (e != cudaSuccess) { free(staged); return report_cuda(e, "psb_build_ex: copy points to host"); }
-        host_pts = staged;
-    }
-    HostLayout h;
-    int rc = psb_host_build(host_pts, n, d, fanout, id_base, flags, &h);
-    free(staged);
-    if (rc != PSB_OK) return rc;
+    const bool dev_in = attr.type == cudaMemoryTypeDevice;
 
     psb_index *ix = new (std::nothrow) psb_index;
     if (!ix) { psb_set_error("psb_build_ex: host allocation failed"); return PSB_ENOMEM; }
     ix->device = dev;
     cudaDeviceGetAttribute(&ix->sm_count, cudaDevAttrMultiProcessorCount, dev);
-    ix->n = h.n; ix->L = h.L; ix->id_base = h.id_base;
-    ix->d = h.d; ix->F = h.F; ix->H = h.H;
-    for (int l = 0; l <= PSB_MAXLVL; ++l) { ix->nlev[l] = h.nlev[l]; ix->level_off[l] = h.level_off[l]; }
-    ix->node_floats = h.total_node_floats;
-    const size_t bp = sizeof(float) * (size_t)(h.L * d * fanout);
-    const size_t bi = sizeof(int32_t) * (size_t)(h.L * fanout);
-    const size_t bn = sizeof(float) * (size_t)h.total_node_floats;
+    ix->n = n; ix->L = shape.L; ix->id_base = id_base;
+    ix->d = d; ix->F = fanout; ix->H = shape.H;
+    for (int l = 0; l <= PSB_MAXLVL; ++l) { ix->nlev[l] = shape.nlev[l]; ix->level_off[l] = shape.level_off[l]; }
+    ix->node_floats = shape.total_node_floats;
+    const size_t bp = sizeof(float) * (size_t)(shape.L * d * fanout);
+    const size_t bi = sizeof(int32_t) * (size_t)(shape.L * fanout);
+    const size_t bn = sizeof(float) * (size_t)shape.total_node_floats;
     if ((e = cudaMalloc((void **)&ix->pts, bp)) != cudaSuccess ||
         (e = cudaMalloc((void **)&ix->ids, bi)) != cudaSuccess ||
-        (e = cudaMalloc((void **)&ix->nodes, bn)) != cudaSuccess ||
-        (e = cudaMemcpy(ix->pts, h.pts, bp, cudaMemcpyHostToDevice)) != cudaSuccess ||
-        (e = cudaMemcpy(ix->ids, h.ids, bi, cudaMemcpyHostToDevice)) != cudaSuccess ||
-        (e = cudaMemcpy(ix->nodes, h.nodes, bn, cudaMemcpyHostToDevice)) != cudaSuccess) {
-        rc = report_cuda(e, "psb_build_ex: upload");
+        (e = cudaMalloc((void **)&ix->nodes, bn)) != cudaSuccess) {
+        rc = report_cuda(e, "psb_build_ex: device allocation");
         index_release(ix);
         return rc;
+    }
+    if (on_gpu) {
+        // NEXT-1: the whole bulk load in CUDA kernels on a private stream
+        cudaStream_t st;
+        if ((e = cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking)) != cudaSuccess) {
+            rc = report_cuda(e, "psb_build_ex: stream");
+            index_release(ix);
+            return rc;
+        }
+        const float *dpts = points;
+        float *staged = nullptr;
+        if (!dev_in) {
+            const size_t bytes = sizeof(float) * (size_t)(n * d);
+            if ((e = cudaMalloc((void **)&staged, bytes)) != cudaSuccess ||
+                (e = cudaMemcpy(staged, points, bytes, cudaMemcpyHostToDevice)) != cudaSuccess) {
+                rc = report_cuda(e, "psb_build_ex: stage points");
+                cudaFree(staged);
+                cudaStreamDestroy(st);
+                index_release(ix);
+                return rc;
+            }
+            dpts = staged;
+        }
+        rc = psb::gpu_bulk_load(dpts, shape, id_base, ix->pts, ix->ids, ix->nodes, st);
+        cudaStreamSynchronize(st);
+        cudaFree(staged);
+        cudaStreamDestroy(st);
+        if (rc != PSB_OK) {
+            index_release(ix);
+            return rc;
+        }
+    } else {
+        const float *host_pts = points;
+        float *staged = nullptr;
+        if (dev_in) {
+            staged = (float *)malloc(sizeof(float) * (size_t)(n * d));
+            if (!staged) { psb_set_error("psb_build_ex: host staging allocation failed"); index_release(ix); return PSB_ENOMEM; }
+            e = cudaMemcpy(staged, points, sizeof(float) * (size_t)(n * d), cudaMemcpyDeviceToHost);
+            if (e != cudaSuccess) { free(staged); rc = report_cuda(e, "psb_build_ex: copy points to host"); index_release(ix); return rc; }
+            host_pts = staged;
+        }
+        HostLayout h;
+        rc = psb_host_build(host_pts, n, d, fanout, id_base, flags, &h);
+        free(staged);
+        if (rc != PSB_OK) { index_release(ix); return rc; }
+        if ((e = cudaMemcpy(ix->pts, h.pts, bp, cudaMemcpyHostToDevice)) != cudaSuccess ||
+            (e = cudaMemcpy(ix->ids, h.ids, bi, cudaMemcpyHostToDevice)) != cudaSuccess ||
+            (e = cudaMemcpy(ix->nodes, h.nodes, bn, cudaMemcpyHostToDevice)) != cudaSuccess) {
+            rc = report_cuda(e, "psb_build_ex: upload");
+            index_release(ix);
+            return rc;
+        }
     }
     ix->device_bytes = (int64_t)(bp + bi + bn);
     // Own pool for per-call scratch; memory stays mapped between calls (a zero

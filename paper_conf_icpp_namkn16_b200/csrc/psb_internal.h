@@ -30,6 +30,19 @@ struct DevIndex {
     int32_t sm_count;                   // of the index's device (launch sizing)
 };
 
+// Level geometry of a packed tree (shared by the host and GPU loaders).
+struct GpuLayoutShape {
+    int64_t n = 0, L = 0;
+    int32_t d = 0, F = 0, H = 0;
+    int64_t nlev[PSB_MAXLVL + 1] = {};
+    int64_t level_off[PSB_MAXLVL + 1] = {};
+    int64_t total_node_floats = 0;
+};
+
+// Validates (n, d, F, id_base, flags) and computes the geometry; PSB_OK or an
+// error code with the message set. Does not read the points.
+int psb_layout_shape(int64_t n, int32_t d, int32_t F, int64_t id_base, uint32_t flags, GpuLayoutShape *s);
+
 struct HostLayout {
     int64_t n = 0, L = 0, id_base = 0;
     int32_t d = 0, F = 0, H = 0;

@@ -305,3 +305,34 @@ def test_host_buffers_and_stats(c2):
         assert np.array_equal(got[0][:, 0] + got[0][:, 3], got[1][:, 0])  # same visits, cache or not
         assert np.array_equal(got[0][:, 1], got[1][:, 1])          # same leaves scanned
         assert (got[0][:, 4] <= got[0][:, 1]).all() and (got[0][:, 5] >= got[0][:, 4]).all()
+
+
+@pytest.mark.parametrize("case", [
+    dict(n=200_000, d=3, F=64, dist="clustered"), dict(n=1, d=2, F=32, dist="uniform"),
+    dict(n=5_001, d=1, F=32, dist="uniform"), dict(n=3_000, d=64, F=512, dist="uniform"),
+    dict(n=100_003, d=16, F=128, dist="clustered"), dict(n=70_000, d=8, F=256, dist="uniform"),
+    dict(n=20_000, d=5, F=32, dist="dups")])
+def test_gpu_bulk_load_matches_host_loader(case):
+    """NEXT-1: the GPU loader (Hilbert keys, CUB radix sort, permutation, MBR
+    levels) builds the same index as the host loader, for host and device input."""
+    psb = _psb()
+    n, d, F = case["n"], case["d"], case["F"]
+    if case["dist"] == "uniform":
+        pts = W.gen_uniform(n, d, 77)
+    elif case["dist"] == "clustered":
+        pts = W.gen_clustered(n, d, 78)
+    else:
+        base = np.random.default_rng(1).integers(0, 6, size=(50, d)).astype(np.float32)
+        pts = base[np.random.default_rng(2).integers(0, 50, size=n)]
+    ref = psb.psb_build_host_blob(pts, F, id_base=11)
+    for src in (pts, torch.from_numpy(pts).cuda()):
+        idx = psb.psb_build_ex(src, F, id_base=11)
+        got = psb.psb_index_export(idx)
+        idx.free()
+        assert np.array_equal(got["ids"], ref["ids"])
+        assert np.array_equal(got["pts"], ref["pts"])
+        for lv in ref["nodes"]:
+            assert np.array_equal(got["nodes"][lv], ref["nodes"][lv]), lv
+    host = psb.psb_build_ex(pts, F, id_base=11, packing=psb.PSB_BUILD_HOST)
+    assert np.array_equal(psb.psb_index_export(host)["ids"], ref["ids"])
+    host.free()

@@ -40,3 +40,13 @@ def test_configs_match_baseline():
     assert W.CONFIGS["C2"].n == 1_000_000 and W.CONFIGS["C2"].k == 32 and W.CONFIGS["C2"].fanout == 64
     assert W.CONFIGS["C3"].q == 100_000 and W.CONFIGS["C3"].d == 8
     assert W.CONFIGS["C5"].n == 512_000_000
+
+
+def test_slabs_are_rows_of_the_full_set():
+    """Data-sharded ranks generate their own slab: it must equal the same rows of
+    the full set (counter-based generator)."""
+    full = W.gen_uniform(10_000, 3, 9)
+    assert np.array_equal(W.gen_uniform(2_500, 3, 9, row0=5_000), full[5_000:7_500])
+    c = W.config("C2", n=20_000)
+    allp = c.points()
+    assert np.array_equal(c.points(n=4_000, row0=12_000), allp[12_000:16_000])

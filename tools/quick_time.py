@@ -13,10 +13,13 @@ def time_it(fn, reps=15):
         s.record(); fn(); e.record(); torch.cuda.synchronize(); ts.append(s.elapsed_time(e))
     return min(ts), float(np.median(ts))
 
-for name in sys.argv[1:] or ["C1", "C2", "C3"]:
+for name in [a for a in sys.argv[1:] if not a.startswith("-")] or ["C1", "C2", "C3"]:
     cfg = W.config(name)
     t0 = time.time(); pts = cfg.points(); qs = cfg.queries(); t1 = time.time()
-    idx = psb.psb_build(pts, cfg.fanout); t2 = time.time()
+    idx = psb.psb_build(pts, cfg.fanout); torch.cuda.synchronize(); t2 = time.time()
+    if "--build" in os.environ.get("QT_FLAGS", ""):
+        th = time.time(); psb.psb_build_ex(pts, cfg.fanout, packing=psb.PSB_BUILD_HOST).free(); th = time.time() - th
+        print(f"{name}: host build {th:.2f}s", flush=True)
     qd = torch.from_numpy(qs).cuda()
     print(f"{name}: gen {t1-t0:.1f}s build {t2-t1:.1f}s info {idx.info()}", flush=True)
     for algo, an in (("psb", 0), ("bnb", 1), ("brute", 2)):

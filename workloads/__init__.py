@@ -63,12 +63,12 @@ def u24(seed: int, start: int, count: int) -> np.ndarray:
     return out
 
 
-def gen_uniform(n: int, d: int, seed: int) -> np.ndarray:
-    """n x d float32 row-major, coordinates u24 in [0, 1)."""
+def gen_uniform(n: int, d: int, seed: int, row0: int = 0) -> np.ndarray:
+    """Rows [row0, row0+n) of the uniform set: n x d float32, coordinates u24 in [0, 1)."""
     out = np.empty(n * d, dtype=np.float32)
     for s in range(0, n * d, _CHUNK):
         c = min(_CHUNK, n * d - s)
-        out[s:s + c] = _u24_range(seed, s, c).astype(np.float32)
+        out[s:s + c] = _u24_range(seed, row0 * d + s, c).astype(np.float32)
     return out.reshape(n, d)
 
 
@@ -85,16 +85,18 @@ def cluster_centres(d: int, seed: int, clusters: int = 100) -> np.ndarray:
 
 
 def gen_clustered(n: int, d: int, seed: int, sigma: float = 160.0,
-                  clusters: int = 100) -> np.ndarray:
-    """n x d float32: `clusters` Gaussian blobs, contiguous id blocks per cluster."""
+                  clusters: int = 100, row0: int = 0, n_total: int | None = None) -> np.ndarray:
+    """Rows [row0, row0+n) of an n_total-point set (default n): `clusters` Gaussian
+    blobs, contiguous id blocks per cluster."""
+    n_total = n if n_total is None else n_total
     c = cluster_centres(d, seed, clusters).astype(np.float64)
-    per = -(-n // clusters)
+    per = -(-n_total // clusters)
     out = np.empty((n, d), dtype=np.float32)
     rows = max(1, _CHUNK // d)
     for s in range(0, n, rows):
         r = min(rows, n - s)
-        m = np.arange(s, s + r) // per
-        g = _normals(seed, s * d, r * d).reshape(r, d)
+        m = np.arange(row0 + s, row0 + s + r) // per
+        g = _normals(seed, (row0 + s) * d, r * d).reshape(r, d)
         out[s:s + r] = (c[m] + sigma * g).astype(np.float32)
     return out
 
@@ -131,11 +133,13 @@ class Config:
     def queries_seed(self) -> int:
         return 0x5053510000 + self.cfg_id
 
-    def points(self, n: int | None = None) -> np.ndarray:
-        n = self.n if n is None else n
+    def points(self, n: int | None = None, row0: int = 0) -> np.ndarray:
+        """Rows [row0, row0+n) of this config's point set (all rows by default;
+        a data-sharded rank asks for its slab)."""
+        n = self.n - row0 if n is None else n
         if self.dist == "uniform":
-            return gen_uniform(n, self.d, self.points_seed)
-        return gen_clustered(n, self.d, self.points_seed, self.sigma)
+            return gen_uniform(n, self.d, self.points_seed, row0)
+        return gen_clustered(n, self.d, self.points_seed, self.sigma, row0=row0, n_total=self.n)
 
     def queries(self, q: int | None = None) -> np.ndarray:
         q = self.q if q is None else q
