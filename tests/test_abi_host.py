@@ -177,6 +177,10 @@ def test_sass_has_no_fused_multiply_add(tmp_path):
                    check=True, capture_output=True)
     cubins = sorted(p for p in os.listdir(tmp_path) if p.endswith(".cubin"))
     assert cubins and all("sm_100a" in c for c in cubins), cubins
+    # the query path (knn_*): distances, bounds, merges. The bulk loader's only
+    # DFMAs are inside the correctly rounded __ddiv_rn routine (Newton steps).
+    cubins = [c for c in cubins if c.startswith("knn_")]
+    assert len(cubins) >= 11, cubins
 
     def scan(c):
         out = subprocess.run(["/usr/local/cuda/bin/nvdisasm", str(tmp_path / c)], capture_output=True,
