@@ -309,23 +309,36 @@ def main():
                          "api": "psb_knn_ex with pinned host buffers (library stages H2D/D2H on the stream)"}
         if args.mode == "data" and world > 1:
             extras["e2e"]["note"] = "local search only (the data-sharded all-gather runs on device buffers)"
-        # single-query latency: launch -> results on the host
-        lat = []
+        # single-query latency: launch -> results on the host,
+        # for PSB (one warp), PSB latency mode (query split over many warps), B&B, brute force
         h1i = torch.empty((1, k), dtype=torch.int32, pin_memory=True)
         h1d = torch.empty((1, k), dtype=torch.float32, pin_memory=True)
-        nl = min(q, 300)
-        for i in range(nl + 10):
-            h1q = hq[i % q:i % q + 1]
-            torch.cuda.synchronize()
-            t0 = time.perf_counter()
-            psb.psb_knn_ex(idx, h1q, k, algo=algo, variant=args.variant, out=(h1i, h1d))
-            stream.synchronize()
-            if i >= 10:
-                lat.append((time.perf_counter() - t0) * 1e6)
-        lat.sort()
-        extras["latency_us"] = {"p50": lat[len(lat) // 2], "p99": lat[int(len(lat) * 0.99)],
-                                "queries": nl, "definition": "one query per call, launch to results "
-                                "in pinned host memory (PAPER.md L835-838 'query response time')"}
+        nl = min(q, 200)
+
+        def lat_of(call, n_lat):
+            lat = []
+            for i in range(n_lat + 5):
+                h1q = hq[i % q:i % q + 1]
+                torch.cuda.synchronize()
+                t0 = time.perf_counter()
+                call(h1q)
+                stream.synchronize()
+                if i >= 5:
+                    lat.append((time.perf_counter() - t0) * 1e6)
+            lat.sort()
+            return {"p50": lat[len(lat) // 2], "p99": lat[min(len(lat) - 1, int(len(lat) * 0.99))],
+                    "queries": n_lat}
+
+        lats = {
+            args.algo: lat_of(lambda x: psb.psb_knn_ex(idx, x, k, algo=algo, variant=args.variant, out=(h1i, h1d)), nl),
+            "psb_split": lat_of(lambda x: psb.psb_knn_split(idx, x, k, parts=0, out=(h1i, h1d)), nl),
+            "bnb": lat_of(lambda x: psb.psb_knn_ex(idx, x, k, algo=psb.PSB_ALGO_BNB, out=(h1i, h1d)), nl),
+            "brute": lat_of(lambda x: psb.psb_knn_ex(idx, x, k, algo=psb.PSB_ALGO_BRUTE, out=(h1i, h1d)),
+                            min(nl, 50)),
+        }
+        extras["latency_us"] = {**lats[args.algo], "by_algo": lats,
+                                "definition": "one query per call, launch to results in pinned host memory "
+                                              "(PAPER.md L835-838 'query response time')"}
         # comparators on the same batch (same timing protocol, fewer steps)
         comp = {}
         for name, a in (("psb", psb.PSB_ALGO_PSB), ("bnb", psb.PSB_ALGO_BNB), ("brute", psb.PSB_ALGO_BRUTE)):

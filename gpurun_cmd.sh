@@ -1,6 +1,14 @@
-timeout 1200 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
-mkdir -p gpurun_out/r01c
-timeout 600 python bench.py > gpurun_out/r01c/bench_C2.json 2> gpurun_out/r01c/bench_C2.err; tail -c 3000 gpurun_out/r01c/bench_C2.json
-timeout 900 python bench.py --config C3 --steps 30 > gpurun_out/r01c/bench_C3.json 2> gpurun_out/r01c/bench_C3.err; tail -c 3000 gpurun_out/r01c/bench_C3.json
-timeout 900 python bench.py --config C4 --steps 20 --no-cpu-baseline > gpurun_out/r01c/bench_C4.json 2> gpurun_out/r01c/bench_C4.err; tail -c 3000 gpurun_out/r01c/bench_C4.json
-timeout 1500 python bench.py --config C5 --mode data --slab 8 --steps 5 --warmup 3 --no-cpu-baseline > gpurun_out/r01c/bench_C5slab8.json 2> gpurun_out/r01c/bench_C5slab8.err; tail -c 3000 gpurun_out/r01c/bench_C5slab8.json; tail -5 gpurun_out/r01c/bench_C5slab8.err
+timeout 1200 python -m pytest tests -m gpu -x -q 2>&1 | tail -5
+python - <<'PY'
+import torch, time, numpy as np, workloads as W, paper_conf_icpp_namkn16_b200 as psb
+for name in ("C2","C3","C4"):
+    cfg=W.config(name); idx=psb.psb_build(cfg.points(), cfg.fanout); qs=cfg.queries(q=64)
+    hq=torch.from_numpy(qs).pin_memory()
+    for parts in (1, 16, 64, 256, 1024, 0):
+        lat=[]
+        for i in range(40):
+            x=hq[i%64:i%64+1]; torch.cuda.synchronize(); t0=time.perf_counter()
+            ids,d=psb.psb_knn_split(idx,x,cfg.k,parts=parts); torch.cuda.synchronize(); lat.append((time.perf_counter()-t0)*1e6)
+        lat=sorted(lat[5:]); print(name,"parts",parts,"p50 us",round(lat[len(lat)//2],1), flush=True)
+    idx.free()
+PY

@@ -100,6 +100,16 @@ int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int6
 int psb_knn(const psb_index *idx, const float *queries, int64_t q, int32_t k,
             int32_t *out_ids, float *out_dists, void *stream);
 
+/* Latency mode of psb_knn (SURVEY.md §8(e) "intra-GPU split"): each query's
+ * leaves are cut into `parts` contiguous ranges, one warp runs PSB on each range,
+ * the warps of a query share their pruning distance through atomicMin, and the
+ * per-range lists are merged on the device. Same results as psb_knn; for small
+ * batches where one warp per query leaves the GPU idle (single-query latency).
+ * parts = 0 picks ~16 warps per SM in total (at least 16 leaves per range);
+ * parts = 1 is psb_knn. */
+int psb_knn_split(const psb_index *idx, const float *queries, int64_t q, int32_t k, int32_t parts,
+                  int32_t *out_ids, float *out_dists, void *stream);
+
 /* The paper's comparison algorithm: classic branch-and-bound kNN (Roussopoulos
  * et al. [17], §III) run data-parallel on the GPU with parent links
  * instead of a stack (§IV-D): children in (MINDIST, index) order,

@@ -31,7 +31,7 @@ FANOUTS = (32, 64, 128, 256, 512)
 
 # every symbol include/psb.h declares (tests check the .so exports all of them)
 EXPORTS = ("psb_build", "psb_build_ex", "psb_knn", "psb_knn_branch_and_bound", "psb_knn_bruteforce",
-           "psb_knn_ex", "psb_knn_stats", "psb_merge_topk", "psb_index_info", "psb_index_export", "psb_build_host_blob",
+           "psb_knn_ex", "psb_knn_stats", "psb_knn_split", "psb_merge_topk", "psb_index_info", "psb_index_export", "psb_build_host_blob",
            "psb_free", "psb_last_error", "psb_version")
 
 if not os.path.exists(LIB_PATH):
@@ -48,6 +48,7 @@ _sig = {
     "psb_knn_branch_and_bound": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp]),
     "psb_knn_bruteforce": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp]),
     "psb_knn_ex": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp, _i32, _u32]),
+    "psb_knn_split": (ctypes.c_int, [_vp, _vp, _i64, _i32, _i32, _vp, _vp, _vp]),
     "psb_knn_stats": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp, _i32, _u32, _vp]),
     "psb_merge_topk": (ctypes.c_int, [_vp, _vp, _i32, _i64, _i32, _vp, _vp, _vp]),
     "psb_index_info": (ctypes.c_int, [_vp, _P(_i64), _P(_i32), _P(_i32), _P(_i64), _P(_i32), _P(_i64)]),
@@ -206,6 +207,14 @@ def psb_knn(index: Index, queries, k: int, stream=None, out=None):
     queries, q, ids, dists = _query_buffers(index, queries, k, out)
     _check(_lib.psb_knn(index.handle, queries.data_ptr(), q, k, ids.data_ptr(), dists.data_ptr(),
                         _stream_handle(stream)), "psb_knn")
+    return ids, dists
+
+
+def psb_knn_split(index: Index, queries, k: int, parts: int = 0, stream=None, out=None):
+    """Latency mode: each query split over `parts` warps (0 = auto)."""
+    queries, q, ids, dists = _query_buffers(index, queries, k, out)
+    _check(_lib.psb_knn_split(index.handle, queries.data_ptr(), q, k, parts, ids.data_ptr(), dists.data_ptr(),
+                              _stream_handle(stream)), "psb_knn_split")
     return ids, dists
 
 

@@ -38,6 +38,85 @@ merge_kernel(const int32_t *__restrict__ ids, const float *__restrict__ dists, i
     T.store(k, lane, out_ids + qi * k, out_dists + qi * k);
 }
 
+// Latency-mode merge: one CTA of MP_WARPS warps per query; warp w takes parts
+// w, w+MP_WARPS, ...; only keys with dist <= the query's final shared pruning
+// distance can belong to the answer, so the rest are dropped before any id load.
+constexpr int MP_WARPS = 32;
+
+template <int KS>
+__global__ void __launch_bounds__(MP_WARPS * 32)
+merge_parts_kernel(const int32_t *__restrict__ ids, const float *__restrict__ dists, const float *__restrict__ gpd,
+                   int parts, int k, int32_t *__restrict__ out_ids, float *__restrict__ out_dists)
+{
+    __shared__ u64 lists[MP_WARPS][KS * 32];
+    __shared__ u64 scratch_all[MP_WARPS][32];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t qi = blockIdx.x;
+    const float lim = __ldg(gpd + qi);
+    TopK<KS> T;
+    T.init();
+    u64 thr = PAD_KEY;
+    constexpr int U = 4;
+    for (int p0 = w; p0 < parts; p0 += MP_WARPS * U) {
+        float dv[U][KS];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int p = p0 + u * MP_WARPS;
+#pragma unroll
+            for (int s = 0; s < KS; ++s) {
+                const int r = s * 32 + lane;
+                dv[u][s] = (p < parts && r < k) ? __ldg(dists + (qi * parts + p) * (int64_t)k + r) : INFINITY;
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int p = p0 + u * MP_WARPS;
+            u64 cand[KS];
+            bool any = false;
+#pragma unroll
+            for (int s = 0; s < KS; ++s) {
+                const int r = s * 32 + lane;
+                const bool ok = p < parts && r < k && dv[u][s] <= lim;
+                cand[s] = ok ? make_key(dv[u][s], __ldg(ids + (qi * parts + p) * (int64_t)k + r)) : ~0ull;
+                any |= ok;
+            }
+            if (__any_sync(FULL, any)) T.template offer<KS>(cand, k, lane, thr, scratch_all[w]);
+        }
+    }
+#pragma unroll
+    for (int s = 0; s < KS; ++s) lists[w][s * 32 + lane] = T.key[s];
+    __syncthreads();
+    if (w == 0) {
+        for (int o = 1; o < MP_WARPS; ++o) {
+            u64 cand[KS];
+#pragma unroll
+            for (int s = 0; s < KS; ++s) cand[s] = s * 32 + lane < k ? lists[o][s * 32 + lane] : ~0ull;
+            T.template offer<KS>(cand, k, lane, thr, scratch_all[0]);
+        }
+        T.store(k, lane, out_ids + qi * k, out_dists + qi * k);
+    }
+}
+
+__global__ void fill_inf(float *__restrict__ p, int64_t n)
+{
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) p[i] = INFINITY;
+}
+
+void init_shared_pd(float *gpd, int64_t nq, cudaStream_t st)
+{
+    fill_inf<<<(unsigned)((nq + 255) / 256), 256, 0, st>>>(gpd, nq);
+}
+
+int launch_merge_parts(const int32_t *ids, const float *dists, const float *gpd, int parts, int64_t nq, int k,
+                       int32_t *oi, float *od, cudaStream_t st)
+{
+    if (k <= 32) merge_parts_kernel<1><<<(unsigned)nq, MP_WARPS * 32, 0, st>>>(ids, dists, gpd, parts, k, oi, od);
+    else if (k <= 64) merge_parts_kernel<2><<<(unsigned)nq, MP_WARPS * 32, 0, st>>>(ids, dists, gpd, parts, k, oi, od);
+    else merge_parts_kernel<4><<<(unsigned)nq, MP_WARPS * 32, 0, st>>>(ids, dists, gpd, parts, k, oi, od);
+    return report_cuda(cudaGetLastError(), "merge_parts kernel launch");
+}
+
 int launch_merge(const int32_t *ids, const float *dists, int parts, int64_t nq, int k, int32_t *oi,
                  float *od, cudaStream_t st)
 {
@@ -50,17 +129,17 @@ int launch_merge(const int32_t *ids, const float *dists, int parts, int64_t nq, 
 
 // Dispatch on d: specialised instantiations for the configs' d, runtime-d otherwise.
 int launch_tree(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool)
+                float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool, int parts)
 {
     int rc = PSB_NOT_INSTANTIATED;
     switch (ix.d) {
-    case 2: rc = launch_tree_v<2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool); break;
-    case 3: rc = launch_tree_v<3>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool); break;
-    case 8: rc = launch_tree_v<8>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool); break;
-    case 16: rc = launch_tree_v<16>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool); break;
+    case 2: rc = launch_tree_v<2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
+    case 3: rc = launch_tree_v<3>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
+    case 8: rc = launch_tree_v<8>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
+    case 16: rc = launch_tree_v<16>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
     default: break;
     }
-    if (rc == PSB_NOT_INSTANTIATED) rc = launch_tree_v<0>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
+    if (rc == PSB_NOT_INSTANTIATED) rc = launch_tree_v<0>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
     return rc == PSB_NOT_INSTANTIATED ? PSB_EUNSUPPORTED : rc;
 }
 

@@ -305,10 +305,161 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
 PSB_TREE_KERNEL(psb_kernel, psb_query)
 PSB_TREE_KERNEL(bnb_kernel, bnb_query)
 
+
+// ---------------------------------------------------------------------------
+// Latency mode (SURVEY.md §8(e) "intra-GPU split"): the leaves of the tree are
+// cut into `parts` contiguous ranges and one warp runs PSB (or B&B) restricted
+// to each range: children whose leaf range misses [lo, hi) are never eligible,
+// `visited` starts at lo-1 and the walk ends when it passes hi-1. The warps of
+// one query share a pruning distance gpd[qi] through atomicMin on its bits
+// (valid: every warp's k-th distance and k-th-MAXDIST bound is an upper bound on
+// the query's true k-th distance, and distances are >= +0 so their bit
+// patterns order like the values). Each warp writes its own sorted list; the
+// lists are merged afterwards (merge_parts_kernel), keeping only keys with
+// dist <= the final gpd. Exact: a point of the true kNN has dist <= d_k <= gpd
+// at all times, so its leaf is never pruned and its warp keeps it.
+__device__ __forceinline__ float shared_pd(const float *g) { return __ldcg(g); }
+__device__ __forceinline__ void publish_pd(float *g, float v)
+{
+    atomicMin(reinterpret_cast<int *>(g), __float_as_int(v));
+}
+
+template <int D, int V, int KS, bool ST>
+__device__ __forceinline__ void psb_part_query(const DevIndex &ix, const float *__restrict__ queries, int64_t qi,
+                                               int part, int parts, int k, int32_t *__restrict__ part_ids,
+                                               float *__restrict__ part_dists, float *__restrict__ gpd,
+                                               const WarpState &ws, bool use_cache, bool use_max, int lane)
+{
+    constexpr int F = 32 * V;
+    constexpr int LOGF = Log2<F>::value;
+    const int H = ix.H;
+    const int L = (int)ix.L;
+    const int chunk = (L + parts - 1) / parts;
+    const int lo = part * chunk, hi = min(lo + chunk, L);
+    TopK<KS> T;
+    T.init();
+    int32_t *oi = part_ids + (qi * parts + part) * (int64_t)k;
+    float *od = part_dists + (qi * parts + part) * (int64_t)k;
+    if (lo >= hi) {
+        T.store(k, lane, oi, od);
+        return;
+    }
+    float *g = gpd + qi;
+    Query<D> q;
+    q.load(queries + qi * ix.d, ix.d, ws.qsmem);
+    for (int l = lane; l <= H; l += 32) ws.cache_node[l] = -1;
+    __syncwarp();
+    u64 thr = PAD_KEY;
+    float pd = shared_pd(g);
+    float published = pd;
+    Stats<ST> S;
+
+    // pass 1 inside the range: greedy descent among children overlapping [lo, hi)
+    int lvl = H, node = 0;
+    while (lvl > 0) {
+        float md[V];
+        internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
+        const int base = node * F, sh = (lvl - 1) * LOGF;
+        const int c_lo = (lo >> sh) - base, c_hi = min((int)ix.nlev[lvl - 1] - base, ((hi - 1) >> sh) - base + 1);
+        u64 best = ~0ull;
+#pragma unroll
+        for (int t = 0; t < V; ++t) {
+            const int c = lane * V + t;
+            if (c >= c_lo && c < c_hi) {
+                const u64 kk = make_key(md[t], c);
+                best = kk < best ? kk : best;
+            }
+        }
+        best = warp_min_u64(best);
+        node = base + (int)(best & 0xffffffffu);
+        --lvl;
+    }
+    const int pass1_lo = node;
+    int pass1_hi = node - 1;
+    int64_t seen = 0;
+    while (seen < k && pass1_hi + 1 < hi) {
+        ++pass1_hi;
+        scan_leaf<D, V, KS, ST>(ix, pass1_hi, q, lane, T, k, thr, S, ws.scratch);
+        const int64_t left = ix.n - (int64_t)pass1_hi * F;
+        seen += left < F ? left : F;
+    }
+    pd = fminf(pd, key_dist(thr));
+    if (pd < published) { if (lane == 0) publish_pd(g, pd); published = pd; }
+
+    lvl = H;
+    node = 0;
+    int visited = lo - 1;
+    while (true) {
+        if (lvl > 0) {
+            float md[V];
+            const float gp = shared_pd(g);                       // issued early, used below
+            internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
+            pd = fminf(pd, gp);
+            const int base = node * F, sh = (lvl - 1) * LOGF;
+            const int c_end = min(min(F, (int)ix.nlev[lvl - 1] - base), ((hi - 1) >> sh) - base + 1);
+            const int c_min = ((visited + 1) >> sh) - base;
+            unsigned mine = 0;
+#pragma unroll
+            for (int t = 0; t < V; ++t) {
+                const int c = lane * V + t;
+                const bool e = c >= c_min && c < c_end && md[t] <= pd;
+                mine |= (unsigned)e << t;
+            }
+            const unsigned bal = __ballot_sync(FULL, mine != 0);
+            if (bal) {
+                const int src = __ffs(bal) - 1;
+                const unsigned m = __shfl_sync(FULL, mine, src);
+                node = base + src * V + (__ffs(m) - 1);
+                --lvl;
+            } else {
+                if (lvl == H) break;
+                visited = max_leaf(ix, lvl, node);
+                if (visited >= hi - 1) break;                    // range exhausted
+                node /= F;
+                ++lvl;
+            }
+        } else {
+            const int j = node;
+            bool changed;
+            if (j >= pass1_lo && j <= pass1_hi) {
+                changed = true;
+            } else {
+                changed = scan_leaf<D, V, KS, ST>(ix, j, q, lane, T, k, thr, S, ws.scratch);
+            }
+            pd = fminf(pd, key_dist(thr));
+            if (pd < published) { if (lane == 0) publish_pd(g, pd); published = pd; }
+            visited = j;
+            if (j >= hi - 1) break;
+            if (changed) {
+                node = j + 1;
+            } else {
+                node = j / F;
+                lvl = 1;
+            }
+        }
+    }
+    T.store(k, lane, oi, od);
+}
+
+template <int D, int V, int KS, bool ST>
+__global__ void __launch_bounds__(WARPS_PER_CTA * 32, PSB_MIN_BLOCKS)
+psb_split_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int parts, int k,
+                 int32_t *__restrict__ part_ids, float *__restrict__ part_dists, float *__restrict__ gpd,
+                 uint32_t variant)
+{
+    extern __shared__ __align__(16) unsigned char smem[];
+    const int lane = threadIdx.x & 31;
+    const int64_t w = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
+    if (w >= nq * parts) return;
+    const WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0);
+    psb_part_query<D, V, KS, ST>(ix, queries, w / parts, (int)(w % parts), parts, k, part_ids, part_dists, gpd, ws,
+                                 !(variant & PSB_VAR_NOCACHE), !(variant & PSB_VAR_NOMAXDIST), lane);
+}
+
 template <int D, int V, int KS>
 static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
                          int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats,
-                         cudaMemPool_t pool)
+                         cudaMemPool_t pool, int parts)
 {
     const size_t smem = WARPS_PER_CTA * WarpSmem::bytes(ix.H, 32 * V, D == 0);
     int64_t blocks = (nq + WARPS_PER_CTA - 1) / WARPS_PER_CTA;
@@ -318,6 +469,34 @@ static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int
     if (smem > 48 * 1024) {
         e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return report_cuda(e, "cudaFuncSetAttribute");
+    }
+    if (parts > 1 && algo == PSB_ALGO_PSB && !stats) {
+        // latency mode: q*parts warps, shared pd per query, then a filtered merge
+        auto sk = psb_split_kernel<D, V, KS, false>;
+        if (smem > 48 * 1024) {
+            e = cudaFuncSetAttribute(sk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+            if (e != cudaSuccess) return report_cuda(e, "cudaFuncSetAttribute");
+        }
+        int32_t *pi = nullptr;
+        float *pdist = nullptr, *gpd = nullptr;
+        const size_t cnt = (size_t)nq * parts * k;
+        if ((e = cudaMallocFromPoolAsync((void **)&pi, cnt * 4, pool, st)) != cudaSuccess ||
+            (e = cudaMallocFromPoolAsync((void **)&pdist, cnt * 4, pool, st)) != cudaSuccess ||
+            (e = cudaMallocFromPoolAsync((void **)&gpd, (size_t)nq * 4, pool, st)) != cudaSuccess) {
+            if (pi) cudaFreeAsync(pi, st);
+            if (pdist) cudaFreeAsync(pdist, st);
+            return report_cuda(e, "cudaMallocFromPoolAsync (split scratch)");
+        }
+        init_shared_pd(gpd, nq, st);                            // +inf per query
+        const int64_t warps = nq * parts;
+        sk<<<(unsigned)((warps + WARPS_PER_CTA - 1) / WARPS_PER_CTA), WARPS_PER_CTA * 32, smem, st>>>(
+            ix, queries, nq, parts, k, pi, pdist, gpd, variant);
+        int rc = report_cuda(cudaGetLastError(), "split kernel launch");
+        if (rc == PSB_OK) rc = launch_merge_parts(pi, pdist, gpd, parts, nq, k, oi, od, st);
+        cudaFreeAsync(pi, st);
+        cudaFreeAsync(pdist, st);
+        cudaFreeAsync(gpd, st);
+        return rc;
     }
     // More queries than resident warps: persistent grid + atomic query queue.
     int per_sm = 0;
@@ -342,28 +521,28 @@ static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int
 template <int D, int V>
 static int launch_tree_ks(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
                           int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats,
-                         cudaMemPool_t pool)
+                         cudaMemPool_t pool, int parts)
 {
-    if (k <= 32) return launch_tree_t<D, V, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
-    if (k <= 64) return launch_tree_t<D, V, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
-    if constexpr (D == 0) return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
+    if (k <= 32) return launch_tree_t<D, V, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
+    if (k <= 64) return launch_tree_t<D, V, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
+    if constexpr (D == 0) return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
     return PSB_NOT_INSTANTIATED;   // k > 64: generic-d kernels (keeps compile time down)
 }
 
 template <int D>
 int launch_tree_v(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
                          int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats,
-                         cudaMemPool_t pool)
+                         cudaMemPool_t pool, int parts)
 {
     switch (ix.F) {
-    case 32: return launch_tree_ks<D, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
-    case 64: return launch_tree_ks<D, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
-    case 128: return launch_tree_ks<D, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
+    case 32: return launch_tree_ks<D, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
+    case 64: return launch_tree_ks<D, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
+    case 128: return launch_tree_ks<D, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
     default: break;
     }
     if constexpr (D == 0) {
-        if (ix.F == 256) return launch_tree_ks<0, 8>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
-        if (ix.F == 512) return launch_tree_ks<0, 16>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool);
+        if (ix.F == 256) return launch_tree_ks<0, 8>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
+        if (ix.F == 512) return launch_tree_ks<0, 16>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
     }
     return PSB_NOT_INSTANTIATED;   // caller falls back to the generic-d kernels
 }

@@ -252,7 +252,7 @@ static bool is_device_ptr(const void *p)
 // staged through stream-ordered device scratch with copies on the same stream.
 static int knn_impl(const char *fn, const psb_index *ix, const float *queries, int64_t q, int32_t k,
                     int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant,
-                    int64_t *stats)
+                    int64_t *stats, int parts = 1)
 {
     g_err[0] = 0;
     int rc = check_query_args(fn, ix, queries, q, k, out_ids, out_dists);
@@ -295,7 +295,7 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
     if (rc == PSB_OK) {
         const DevIndex v = dev_view(ix);
         rc = algo == PSB_ALGO_BRUTE ? psb::launch_brute(v, dq, q, k, di, dd, st, ix->sm_count, ix->pool)
-                                    : psb::launch_tree(algo, v, dq, q, k, di, dd, st, variant, stats, ix->pool);
+                                    : psb::launch_tree(algo, v, dq, q, k, di, dd, st, variant, stats, ix->pool, parts);
     }
     if (ho) {
         if (rc == PSB_OK && ((e = cudaMemcpyAsync(out_ids, di, bo, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||
@@ -323,6 +323,23 @@ int psb_knn_stats(const psb_index *ix, const float *queries, int64_t q, int32_t 
         return PSB_EINVAL;
     }
     return knn_impl("psb_knn_stats", ix, queries, q, k, out_ids, out_dists, stream, algo, variant, stats);
+}
+
+int psb_knn_split(const psb_index *ix, const float *queries, int64_t q, int32_t k, int32_t parts,
+                  int32_t *out_ids, float *out_dists, void *stream)
+{
+    if (parts < 0) { psb_set_error("psb_knn_split: parts=%d < 0", parts); return PSB_EINVAL; }
+    if (ix && parts == 0) {
+        // auto: about 16 warps per SM in total, at least 16 leaves per part
+        const int64_t target = (int64_t)ix->sm_count * 16;
+        int64_t p = q > 0 ? target / q : 1;
+        const int64_t pmax = ix->L / 16;
+        if (p > pmax) p = pmax;
+        parts = (int32_t)(p < 1 ? 1 : p);
+    }
+    if (ix && parts > ix->L) parts = (int32_t)ix->L;
+    return knn_impl("psb_knn_split", ix, queries, q, k, out_ids, out_dists, stream, PSB_ALGO_PSB, 0, nullptr,
+                    parts < 1 ? 1 : parts);
 }
 
 int psb_knn(const psb_index *ix, const float *queries, int64_t q, int32_t k, int32_t *out_ids,

@@ -12,8 +12,9 @@ int report_cuda(cudaError_t e, const char *what);
 // PSB_ALGO_PSB or PSB_ALGO_BNB, one warp per query (knn_tree.cu).
 // `stats` (nullable, device [nq][4] int64): per query {internal node fetches,
 // leaf scans, id loads, path-cache hits}.
+// parts > 1 (PSB only): latency mode, each query's leaves split over `parts` warps.
 int launch_tree(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool);
+                float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool, int parts);
 
 // Exhaustive scan of all points (knn_brute.cu). Splits the point set into
 // chunks when there are too few queries to fill the GPU and merges the partial
@@ -26,7 +27,13 @@ int launch_brute(const DevIndex &ix, const float *queries, int64_t nq, int k, in
 constexpr int PSB_NOT_INSTANTIATED = 1;
 template <int D>
 int launch_tree_v(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                  float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool);
+                  float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool, int parts);
+
+// Latency-mode helpers (knn_merge.cu): shared pruning distances to +inf, and the
+// filtered merge of [nq][parts][k] per-part lists.
+void init_shared_pd(float *gpd, int64_t nq, cudaStream_t st);
+int launch_merge_parts(const int32_t *ids, const float *dists, const float *gpd, int parts, int64_t nq, int k,
+                       int32_t *oi, float *od, cudaStream_t st);
 template <int D>
 int launch_brute_v(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi, float *od,
                    cudaStream_t st, int sm, cudaMemPool_t pool);

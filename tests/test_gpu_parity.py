@@ -336,3 +336,29 @@ def test_gpu_bulk_load_matches_host_loader(case):
     host = psb.psb_build_ex(pts, F, id_base=11, packing=psb.PSB_BUILD_HOST)
     assert np.array_equal(psb.psb_index_export(host)["ids"], ref["ids"])
     host.free()
+
+
+@pytest.mark.parametrize("nq,parts", [(1, 0), (1, 7), (3, 64), (64, 0), (1000, 2), (200, 1)])
+def test_split_latency_mode(c2, nq, parts):
+    """psb_knn_split (each query's leaves over `parts` warps, shared pruning
+    distance, filtered merge) returns exactly psb_knn's rows."""
+    psb = _psb()
+    cfg, pts, qs, idx, exp = c2
+    sl = slice(100, 100 + nq)
+    ids, d = psb.psb_knn_split(idx, torch.from_numpy(qs[sl].copy()).cuda(), cfg.k, parts=parts)
+    torch.cuda.synchronize()
+    assert_same((ids.cpu().numpy(), d.cpu().numpy()), (exp[0][sl], exp[1][sl]), f"split nq={nq} parts={parts}")
+
+
+@pytest.mark.parametrize("case", [dict(n=5, d=3, F=32, k=8, parts=4), dict(n=40_000, d=16, F=128, k=100, parts=0),
+                                  dict(n=30_000, d=5, F=64, k=1, parts=13), dict(n=9_000, d=2, F=32, k=64, parts=300)])
+def test_split_edges(case):
+    psb = _psb()
+    rng = np.random.default_rng(case["n"])
+    pts = (rng.normal(size=(case["n"], case["d"])) * 10).astype(np.float32)
+    qs = (rng.normal(size=(5, case["d"])) * 12).astype(np.float32)
+    idx = psb.psb_build(pts, case["F"])
+    ids, d = psb.psb_knn_split(idx, torch.from_numpy(qs).cuda(), case["k"], parts=case["parts"])
+    torch.cuda.synchronize()
+    assert_same((ids.cpu().numpy(), d.cpu().numpy()), oracle.knn_bruteforce(pts, qs, case["k"]), str(case))
+    idx.free()
