@@ -1,0 +1,23 @@
+"""Small runs of every kernel family for compute-sanitizer (memcheck, racecheck,
+synccheck, initcheck): C1-shaped and C2-sampled inputs, all algorithms, latency
+mode, stats, merge and the GPU bulk loader."""
+import os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, torch
+import paper_conf_icpp_namkn16_b200 as psb
+import workloads as W
+
+for name, n, q in (("C1", None, 100), ("C2", 100_000, 64)):
+    cfg = W.config(name)
+    pts = cfg.points(n=n)
+    qd = torch.from_numpy(cfg.queries(q=q)).cuda()
+    idx = psb.psb_build(pts, cfg.fanout)
+    for algo in (0, 1, 2):
+        psb.psb_knn_ex(idx, qd, cfg.k, algo=algo)
+    psb.psb_knn_stats(idx, qd, cfg.k, algo=0)
+    psb.psb_knn_split(idx, qd[:4], cfg.k, parts=16)
+    ids, d = psb.psb_knn(idx, qd, cfg.k)
+    psb.psb_merge_topk(torch.stack([ids, ids]), torch.stack([d, d]), cfg.k)
+    torch.cuda.synchronize()
+    idx.free()
+print("sanitize workload done")
