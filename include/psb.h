@@ -62,6 +62,14 @@ enum { PSB_PACK_HILBERT = 0, PSB_PACK_STR = 1 };
  * kernels; NEXT-1); PSB_BUILD_HOST forces the host (OpenMP) loader. STR always
  * runs on the host. Both loaders produce the same index. */
 #define PSB_BUILD_HOST 0x100u
+/* Node-shape flag (OR into psb_build_ex `flags`): SS-tree bounding spheres
+ * instead of MBRs (the paper's own index, §II-C; NEXT-2). Each internal
+ * node stores its children's spheres as rows centre[d][fanout] then
+ * radius[fanout], built bottom-up by parallel Ritter (Alg. 2) on the
+ * GPU with radii rounded up so every point is contained. Query bounds use
+ * directed rounding plus a relative margin, so results stay exact. GPU Hilbert
+ * loader only (not with PSB_BUILD_HOST / PSB_PACK_STR). */
+#define PSB_NODE_SPHERE 0x200u
 
 #define PSB_KMAX 128          /* largest k served by the warp top-k (4 keys per lane) */
 #define PSB_DMAX 64           /* largest dimensionality                               */
@@ -164,12 +172,14 @@ int psb_index_info(const psb_index *idx, int64_t *n, int32_t *d, int32_t *fanout
 
 /* Copy the index's flat arrays to host memory (tests, replicas). Layout of the
  * exported blob (all little-endian):
- *   int64 header[8] = {n, d, fanout, leaves L, levels H, id_base, total_nodes, 0}
+ *   int64 header[8] = {n, d, fanout, leaves L, levels H, id_base, total_nodes, sphere}
  *   int64 nodes_per_level[H+1]            (level 0 = L leaves)
  *   float pts[L][d][fanout]               (leaf-blocked SoA; pad slots +inf)
  *   int32 ids[L][fanout]                  (pad slots -1)
  *   float nodes: for level 1..H, nodes_per_level[l] blocks of [d][2][fanout]
- *                (row 2j = lo of dim j, row 2j+1 = hi; empty slots lo=+inf, hi=-inf)
+ *                (row 2j = lo of dim j, row 2j+1 = hi; empty slots lo=+inf, hi=-inf),
+ *                or for sphere indexes blocks of [d+1][fanout] (centre rows, then
+ *                the radius row; empty slots centre +inf, radius 0)
  * If host_buf is NULL or cap is too small, only *used is written (required size)
  * and PSB_EINVAL is returned when host_buf is non-NULL. Synchronous. */
 int psb_index_export(const psb_index *idx, void *host_buf, int64_t cap, int64_t *used);

@@ -24,6 +24,7 @@ LIB_PATH = os.environ.get("PSB_LIB_PATH") or os.path.join(_HERE, "libpsb.so")   
 PSB_OK, PSB_EINVAL, PSB_ENOMEM, PSB_ECUDA, PSB_EUNSUPPORTED = 0, -1, -2, -3, -4
 PSB_PACK_HILBERT, PSB_PACK_STR = 0, 1
 PSB_BUILD_HOST = 0x100
+PSB_NODE_SPHERE = 0x200
 PSB_ALGO_PSB, PSB_ALGO_BNB, PSB_ALGO_BRUTE = 0, 1, 2
 PSB_VAR_NOCACHE, PSB_VAR_NOMAXDIST = 1, 2
 PSB_KMAX, PSB_DMAX = 128, 64
@@ -249,7 +250,7 @@ def psb_merge_topk(ids, dists, k: int, stream=None, out=None):
 
 def _parse_blob(buf: np.ndarray) -> dict:
     hdr = buf[:64].view(np.int64)
-    n, d, F, L, H, id_base, total = (int(x) for x in hdr[:7])
+    n, d, F, L, H, id_base, total, sphere = (int(x) for x in hdr[:8])
     o = 64
     nlev = buf[o:o + 8 * (H + 1)].view(np.int64).copy()
     o += 8 * (H + 1)
@@ -260,9 +261,13 @@ def _parse_blob(buf: np.ndarray) -> dict:
     levels = {}
     for lv in range(1, H + 1):
         cnt = int(nlev[lv])
-        levels[lv] = buf[o:o + 4 * cnt * 2 * d * F].view(np.float32).reshape(cnt, d, 2, F)
-        o += 4 * cnt * 2 * d * F
-    return {"n": n, "d": d, "fanout": F, "leaves": L, "levels": H, "id_base": id_base,
+        if sphere:
+            levels[lv] = buf[o:o + 4 * cnt * (d + 1) * F].view(np.float32).reshape(cnt, d + 1, F)
+            o += 4 * cnt * (d + 1) * F
+        else:
+            levels[lv] = buf[o:o + 4 * cnt * 2 * d * F].view(np.float32).reshape(cnt, d, 2, F)
+            o += 4 * cnt * 2 * d * F
+    return {"n": n, "d": d, "fanout": F, "leaves": L, "levels": H, "id_base": id_base, "sphere": bool(sphere),
             "total_nodes": total, "nlev": nlev, "pts": pts, "ids": ids, "nodes": levels}
 
 

@@ -116,30 +116,13 @@ static int launch_brute_t(const DevIndex &ix, const float *queries, int64_t nq, 
 }
 
 template <int D, int V>
-static int launch_brute_ks(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
+int launch_brute_ks(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
                            float *od, cudaStream_t st, int sm, cudaMemPool_t pool)
 {
     if (k <= 32) return launch_brute_t<D, V, 1>(ix, queries, nq, k, oi, od, st, sm, pool);
     if (k <= 64) return launch_brute_t<D, V, 2>(ix, queries, nq, k, oi, od, st, sm, pool);
     if constexpr (D == 0) return launch_brute_t<D, V, 4>(ix, queries, nq, k, oi, od, st, sm, pool);
     return PSB_NOT_INSTANTIATED;   // k > 64: generic-d kernels
-}
-
-template <int D>
-int launch_brute_v(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                          float *od, cudaStream_t st, int sm, cudaMemPool_t pool)
-{
-    switch (ix.F) {
-    case 32: return launch_brute_ks<D, 1>(ix, queries, nq, k, oi, od, st, sm, pool);
-    case 64: return launch_brute_ks<D, 2>(ix, queries, nq, k, oi, od, st, sm, pool);
-    case 128: return launch_brute_ks<D, 4>(ix, queries, nq, k, oi, od, st, sm, pool);
-    default: break;
-    }
-    if constexpr (D == 0) {
-        if (ix.F == 256) return launch_brute_ks<0, 8>(ix, queries, nq, k, oi, od, st, sm, pool);
-        if (ix.F == 512) return launch_brute_ks<0, 16>(ix, queries, nq, k, oi, od, st, sm, pool);
-    }
-    return PSB_NOT_INSTANTIATED;
 }
 
 }  // namespace psb

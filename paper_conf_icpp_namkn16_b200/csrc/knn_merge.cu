@@ -127,19 +127,29 @@ int launch_merge(const int32_t *ids, const float *dists, int parts, int64_t nq, 
     return report_cuda(cudaGetLastError(), "merge kernel launch");
 }
 
-// Dispatch on d: specialised instantiations for the configs' d, runtime-d otherwise.
+// Dispatch on (d, fanout): the configs' specialisations, runtime-d otherwise.
+#define PSB_SPECIALISED(X) X(2, 1) X(3, 2) X(3, 4) X(8, 4) X(16, 4)
+
 int launch_tree(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
                 float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool, int parts)
 {
     int rc = PSB_NOT_INSTANTIATED;
-    switch (ix.d) {
-    case 2: rc = launch_tree_v<2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
-    case 3: rc = launch_tree_v<3>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
-    case 8: rc = launch_tree_v<8>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
-    case 16: rc = launch_tree_v<16>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
-    default: break;
+    const int V = ix.F / 32;
+#define TRY(DD, VV)                                                                                  \
+    if (rc == PSB_NOT_INSTANTIATED && ix.d == DD && V == VV)                                        \
+        rc = launch_tree_ks<DD, VV>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
+    PSB_SPECIALISED(TRY)
+#undef TRY
+    if (rc == PSB_NOT_INSTANTIATED) {
+        switch (V) {
+        case 1: rc = launch_tree_ks<0, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
+        case 2: rc = launch_tree_ks<0, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
+        case 4: rc = launch_tree_ks<0, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
+        case 8: rc = launch_tree_ks<0, 8>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
+        case 16: rc = launch_tree_ks<0, 16>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
+        default: break;
+        }
     }
-    if (rc == PSB_NOT_INSTANTIATED) rc = launch_tree_v<0>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
     return rc == PSB_NOT_INSTANTIATED ? PSB_EUNSUPPORTED : rc;
 }
 
@@ -147,14 +157,22 @@ int launch_brute(const DevIndex &ix, const float *queries, int64_t nq, int k, in
                  cudaStream_t st, int sm_count, cudaMemPool_t pool)
 {
     int rc = PSB_NOT_INSTANTIATED;
-    switch (ix.d) {
-    case 2: rc = launch_brute_v<2>(ix, queries, nq, k, oi, od, st, sm_count, pool); break;
-    case 3: rc = launch_brute_v<3>(ix, queries, nq, k, oi, od, st, sm_count, pool); break;
-    case 8: rc = launch_brute_v<8>(ix, queries, nq, k, oi, od, st, sm_count, pool); break;
-    case 16: rc = launch_brute_v<16>(ix, queries, nq, k, oi, od, st, sm_count, pool); break;
-    default: break;
+    const int V = ix.F / 32;
+#define TRY(DD, VV)                                                                                  \
+    if (rc == PSB_NOT_INSTANTIATED && ix.d == DD && V == VV)                                        \
+        rc = launch_brute_ks<DD, VV>(ix, queries, nq, k, oi, od, st, sm_count, pool);
+    PSB_SPECIALISED(TRY)
+#undef TRY
+    if (rc == PSB_NOT_INSTANTIATED) {
+        switch (V) {
+        case 1: rc = launch_brute_ks<0, 1>(ix, queries, nq, k, oi, od, st, sm_count, pool); break;
+        case 2: rc = launch_brute_ks<0, 2>(ix, queries, nq, k, oi, od, st, sm_count, pool); break;
+        case 4: rc = launch_brute_ks<0, 4>(ix, queries, nq, k, oi, od, st, sm_count, pool); break;
+        case 8: rc = launch_brute_ks<0, 8>(ix, queries, nq, k, oi, od, st, sm_count, pool); break;
+        case 16: rc = launch_brute_ks<0, 16>(ix, queries, nq, k, oi, od, st, sm_count, pool); break;
+        default: break;
+        }
     }
-    if (rc == PSB_NOT_INSTANTIATED) rc = launch_brute_v<0>(ix, queries, nq, k, oi, od, st, sm_count, pool);
     return rc == PSB_NOT_INSTANTIATED ? PSB_EUNSUPPORTED : rc;
 }
 

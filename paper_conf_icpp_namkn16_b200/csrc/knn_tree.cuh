@@ -44,7 +44,7 @@ __device__ __forceinline__ WarpState warp_state(unsigned char *smem, int H, int 
 // A node already cached at its level is not fetched again: MINDIST is a pure
 // function of (query, node), and its k-th-MAXDIST bound was applied when it was
 // first fetched (re-applying it could not lower pd further).
-template <int D, int V>
+template <int D, int V, bool SPH>
 __device__ __forceinline__ bool internal_md(const DevIndex &ix, int lvl, int node,
                                             const Query<D> &q, int lane, const WarpState &ws,
                                             bool use_cache, bool use_max, int k, float &pd,
@@ -57,13 +57,15 @@ __device__ __forceinline__ bool internal_md(const DevIndex &ix, int lvl, int nod
         for (int t = 0; t < V; ++t) md[t] = cm[t];
         return false;
     }
-    const float *blk = ix.nodes + ix.level_off[lvl] + (int64_t)node * (2 * ix.d * F);
+    const float *blk = ix.nodes + ix.level_off[lvl] + (int64_t)node * ix.blk_floats;
     float Md[V];
     if (use_max) {
-        node_bounds<D, V, true>(blk, q, ix.d, lane, md, Md);
+        if constexpr (SPH) sphere_bounds<D, V, true>(blk, q, ix.d, lane, md, Md);
+        else node_bounds<D, V, true>(blk, q, ix.d, lane, md, Md);
         pd = kth_bound<V>(Md, k, pd);                    // Alg. 1 l.13-15
     } else {
-        node_bounds<D, V, false>(blk, q, ix.d, lane, md, Md);
+        if constexpr (SPH) sphere_bounds<D, V, false>(blk, q, ix.d, lane, md, Md);
+        else node_bounds<D, V, false>(blk, q, ix.d, lane, md, Md);
     }
     if (use_cache) {
 #pragma unroll
@@ -89,7 +91,7 @@ struct Log2 {
 };
 
 // PSB for query qi, executed by one warp (Alg. 1 with the readings of DESIGN.md §2).
-template <int D, int V, int KS, bool ST>
+template <int D, int V, int KS, bool ST, bool SPH>
 __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__restrict__ queries, int64_t qi,
                                           int k, int32_t *__restrict__ out_ids, float *__restrict__ out_dists,
                                           int64_t *__restrict__ stats, const WarpState &ws, bool use_cache,
@@ -116,7 +118,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     int node = 0;
     while (lvl > 0) {
         float md[V];
-        S.node(internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
+        S.node(internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
         const int base = node * F, nb = (int)ix.nlev[lvl - 1];
         u64 best = ~0ull;
 #pragma unroll
@@ -152,7 +154,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     while (true) {
         if (lvl > 0) {
             float md[V];
-            S.node(internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
+            S.node(internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
             // S6: eligible(c) = MINDIST <= pd (R5) and unvisited leaves below (R8).
             // Subtree leaf ranges are contiguous and increasing in c, so
             // maxLeaf(child c) > visited  <=>  visited+1 < L  and
@@ -207,7 +209,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
 // Stackless B&B: at an internal node take the next child in
 // (MINDIST, index) order after the one we returned from, among those with
 // MINDIST <= pd; a leaf always returns to its parent.
-template <int D, int V, int KS, bool ST>
+template <int D, int V, int KS, bool ST, bool SPH>
 __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__restrict__ queries, int64_t qi,
                                           int k, int32_t *__restrict__ out_ids, float *__restrict__ out_dists,
                                           int64_t *__restrict__ stats, const WarpState &ws, bool use_cache,
@@ -232,7 +234,7 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
     while (true) {
         if (lvl > 0) {
             float md[V];
-            S.node(internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
+            S.node(internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
             u64 from_key = 0;
             if (from_c >= 0) {
                 float v = md[0];
@@ -278,7 +280,7 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
 // CTAs as fit on the GPU) and each warp takes the next query from an atomic
 // counter when it finishes one, so a long query never holds an idle block.
 #define PSB_TREE_KERNEL(NAME, BODY)                                                                  \
-    template <int D, int V, int KS, bool ST>                                                          \
+    template <int D, int V, int KS, bool ST, bool SPH>                                                \
     __global__ void __launch_bounds__(WARPS_PER_CTA * 32, PSB_MIN_BLOCKS)                            \
     NAME(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,                          \
          int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant,             \
@@ -297,7 +299,7 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
                 qi = (int64_t)__shfl_sync(FULL, v, 0);                                                \
             }                                                                                         \
             if (qi >= nq) break;                                                                      \
-            BODY<D, V, KS, ST>(ix, queries, qi, k, out_ids, out_dists, stats, ws, use_cache, use_max, lane); \
+            BODY<D, V, KS, ST, SPH>(ix, queries, qi, k, out_ids, out_dists, stats, ws, use_cache, use_max, lane); \
             if (!queue) break;                                                                        \
         }                                                                                             \
     }
@@ -324,7 +326,7 @@ __device__ __forceinline__ void publish_pd(float *g, float v)
     atomicMin(reinterpret_cast<int *>(g), __float_as_int(v));
 }
 
-template <int D, int V, int KS, bool ST>
+template <int D, int V, int KS, bool ST, bool SPH>
 __device__ __forceinline__ void psb_part_query(const DevIndex &ix, const float *__restrict__ queries, int64_t qi,
                                                int part, int parts, int k, int32_t *__restrict__ part_ids,
                                                float *__restrict__ part_dists, float *__restrict__ gpd,
@@ -358,7 +360,7 @@ __device__ __forceinline__ void psb_part_query(const DevIndex &ix, const float *
     int lvl = H, node = 0;
     while (lvl > 0) {
         float md[V];
-        internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
+        internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
         const int base = node * F, sh = (lvl - 1) * LOGF;
         const int c_lo = (lo >> sh) - base, c_hi = min((int)ix.nlev[lvl - 1] - base, ((hi - 1) >> sh) - base + 1);
         u64 best = ~0ull;
@@ -393,7 +395,7 @@ __device__ __forceinline__ void psb_part_query(const DevIndex &ix, const float *
         if (lvl > 0) {
             float md[V];
             const float gp = shared_pd(g);                       // issued early, used below
-            internal_md<D, V>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
+            internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
             pd = fminf(pd, gp);
             const int base = node * F, sh = (lvl - 1) * LOGF;
             const int c_end = min(min(F, (int)ix.nlev[lvl - 1] - base), ((hi - 1) >> sh) - base + 1);
@@ -441,7 +443,7 @@ __device__ __forceinline__ void psb_part_query(const DevIndex &ix, const float *
     T.store(k, lane, oi, od);
 }
 
-template <int D, int V, int KS, bool ST>
+template <int D, int V, int KS, bool ST, bool SPH>
 __global__ void __launch_bounds__(WARPS_PER_CTA * 32, PSB_MIN_BLOCKS)
 psb_split_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int parts, int k,
                  int32_t *__restrict__ part_ids, float *__restrict__ part_dists, float *__restrict__ gpd,
@@ -452,7 +454,7 @@ psb_split_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int
     const int64_t w = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
     if (w >= nq * parts) return;
     const WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0);
-    psb_part_query<D, V, KS, ST>(ix, queries, w / parts, (int)(w % parts), parts, k, part_ids, part_dists, gpd, ws,
+    psb_part_query<D, V, KS, ST, SPH>(ix, queries, w / parts, (int)(w % parts), parts, k, part_ids, part_dists, gpd, ws,
                                  !(variant & PSB_VAR_NOCACHE), !(variant & PSB_VAR_NOMAXDIST), lane);
 }
 
@@ -463,8 +465,24 @@ static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int
 {
     const size_t smem = WARPS_PER_CTA * WarpSmem::bytes(ix.H, 32 * V, D == 0);
     int64_t blocks = (nq + WARPS_PER_CTA - 1) / WARPS_PER_CTA;
-    auto kern = algo == PSB_ALGO_PSB ? (stats ? psb_kernel<D, V, KS, true> : psb_kernel<D, V, KS, false>)
-                                     : (stats ? bnb_kernel<D, V, KS, true> : bnb_kernel<D, V, KS, false>);
+    // Counting (stats) kernels are instantiated for the generic-d path only: the
+    // traversal, hence every counter, does not depend on the d specialisation.
+    using Kern = void (*)(DevIndex, const float *, int64_t, int, int32_t *, float *, uint32_t, int64_t *,
+                          unsigned long long *);
+    Kern kern;
+    const bool psbk = algo == PSB_ALGO_PSB;
+    if constexpr (D == 0) {
+        if (ix.sphere)
+            kern = psbk ? (stats ? psb_kernel<D, V, KS, true, true> : psb_kernel<D, V, KS, false, true>)
+                        : (stats ? bnb_kernel<D, V, KS, true, true> : bnb_kernel<D, V, KS, false, true>);
+        else
+            kern = psbk ? (stats ? psb_kernel<D, V, KS, true, false> : psb_kernel<D, V, KS, false, false>)
+                        : (stats ? bnb_kernel<D, V, KS, true, false> : bnb_kernel<D, V, KS, false, false>);
+    } else {
+        if (stats) return PSB_NOT_INSTANTIATED;
+        if (ix.sphere) kern = psbk ? psb_kernel<D, V, KS, false, true> : bnb_kernel<D, V, KS, false, true>;
+        else kern = psbk ? psb_kernel<D, V, KS, false, false> : bnb_kernel<D, V, KS, false, false>;
+    }
     cudaError_t e;
     if (smem > 48 * 1024) {
         e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -472,7 +490,7 @@ static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int
     }
     if (parts > 1 && algo == PSB_ALGO_PSB && !stats) {
         // latency mode: q*parts warps, shared pd per query, then a filtered merge
-        auto sk = psb_split_kernel<D, V, KS, false>;
+        auto sk = ix.sphere ? psb_split_kernel<D, V, KS, false, true> : psb_split_kernel<D, V, KS, false, false>;
         if (smem > 48 * 1024) {
             e = cudaFuncSetAttribute(sk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
             if (e != cudaSuccess) return report_cuda(e, "cudaFuncSetAttribute");
@@ -519,7 +537,7 @@ static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int
 }
 
 template <int D, int V>
-static int launch_tree_ks(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
+int launch_tree_ks(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
                           int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats,
                          cudaMemPool_t pool, int parts)
 {
@@ -527,24 +545,6 @@ static int launch_tree_ks(int algo, const DevIndex &ix, const float *queries, in
     if (k <= 64) return launch_tree_t<D, V, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
     if constexpr (D == 0) return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
     return PSB_NOT_INSTANTIATED;   // k > 64: generic-d kernels (keeps compile time down)
-}
-
-template <int D>
-int launch_tree_v(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
-                         int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats,
-                         cudaMemPool_t pool, int parts)
-{
-    switch (ix.F) {
-    case 32: return launch_tree_ks<D, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
-    case 64: return launch_tree_ks<D, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
-    case 128: return launch_tree_ks<D, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
-    default: break;
-    }
-    if constexpr (D == 0) {
-        if (ix.F == 256) return launch_tree_ks<0, 8>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
-        if (ix.F == 512) return launch_tree_ks<0, 16>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
-    }
-    return PSB_NOT_INSTANTIATED;   // caller falls back to the generic-d kernels
 }
 
 }  // namespace psb

@@ -47,6 +47,7 @@ struct psb_index {
     int32_t *ids = nullptr;
     float *nodes = nullptr;
     int64_t device_bytes = 0;
+    int32_t sphere = 0, blk_floats = 0;
     cudaMemPool_t pool = nullptr;   // stream-ordered scratch (host-buffer staging, brute-force partials)
 };
 
@@ -86,6 +87,8 @@ static DevIndex dev_view(const psb_index *ix)
     v.d = ix->d;
     v.F = ix->F;
     v.sm_count = ix->sm_count;
+    v.sphere = ix->sphere;
+    v.blk_floats = ix->blk_floats;
     return v;
 }
 
@@ -112,7 +115,13 @@ int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int6
     GpuLayoutShape shape;
     int rc = psb_layout_shape(n, d, fanout, id_base, flags, &shape);
     if (rc != PSB_OK) return rc;
-    const bool on_gpu = (flags & ~(uint32_t)PSB_BUILD_HOST) == PSB_PACK_HILBERT && !(flags & PSB_BUILD_HOST);
+    const bool sphere = (flags & PSB_NODE_SPHERE) != 0;
+    const bool on_gpu = (flags & ~(uint32_t)(PSB_BUILD_HOST | PSB_NODE_SPHERE)) == PSB_PACK_HILBERT &&
+                        !(flags & PSB_BUILD_HOST);
+    if (sphere && !on_gpu) {
+        psb_set_error("psb_build_ex: PSB_NODE_SPHERE needs the GPU Hilbert loader");
+        return PSB_EUNSUPPORTED;
+    }
     cudaPointerAttributes attr;
     e = cudaPointerGetAttributes(&attr, points);
     if (e != cudaSuccess) {
@@ -129,6 +138,8 @@ int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int6
     ix->d = d; ix->F = fanout; ix->H = shape.H;
     for (int l = 0; l <= PSB_MAXLVL; ++l) { ix->nlev[l] = shape.nlev[l]; ix->level_off[l] = shape.level_off[l]; }
     ix->node_floats = shape.total_node_floats;
+    ix->sphere = shape.sphere;
+    ix->blk_floats = shape.blk_floats;
     const size_t bp = sizeof(float) * (size_t)(shape.L * d * fanout);
     const size_t bi = sizeof(int32_t) * (size_t)(shape.L * fanout);
     const size_t bn = sizeof(float) * (size_t)shape.total_node_floats;
@@ -161,7 +172,7 @@ int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int6
             }
             dpts = staged;
         }
-        rc = psb::gpu_bulk_load(dpts, shape, id_base, ix->pts, ix->ids, ix->nodes, st);
+        rc = psb::gpu_bulk_load(dpts, shape, id_base, ix->pts, ix->ids, ix->nodes, st, sphere);
         cudaStreamSynchronize(st);
         cudaFree(staged);
         cudaStreamDestroy(st);
@@ -395,11 +406,11 @@ static int64_t blob_size(int64_t L, int32_t d, int32_t F, int32_t H, int64_t nod
 }
 
 static void blob_header(char *buf, int64_t n, int32_t d, int32_t F, int64_t L, int32_t H, int64_t id_base,
-                        const int64_t *nlev)
+                        const int64_t *nlev, int32_t sphere = 0)
 {
     int64_t total = 0;
     for (int l = 1; l <= H; ++l) total += nlev[l];
-    int64_t hdr[8] = {n, d, F, L, H, id_base, total, 0};
+    int64_t hdr[8] = {n, d, F, L, H, id_base, total, sphere};
     memcpy(buf, hdr, sizeof hdr);
     memcpy(buf + sizeof hdr, nlev, 8 * (size_t)(H + 1));
 }
@@ -412,7 +423,7 @@ int psb_index_export(const psb_index *ix, void *host_buf, int64_t cap, int64_t *
     if (!host_buf) return PSB_OK;
     if (cap < need) { psb_set_error("psb_index_export: cap %lld < %lld", (long long)cap, (long long)need); return PSB_EINVAL; }
     char *b = (char *)host_buf;
-    blob_header(b, ix->n, ix->d, ix->F, ix->L, ix->H, ix->id_base, ix->nlev);
+    blob_header(b, ix->n, ix->d, ix->F, ix->L, ix->H, ix->id_base, ix->nlev, ix->sphere);
     char *p = b + 64 + 8 * (ix->H + 1);
     const size_t bp = 4 * (size_t)(ix->L * ix->d * ix->F), bi = 4 * (size_t)(ix->L * ix->F);
     cudaError_t e;

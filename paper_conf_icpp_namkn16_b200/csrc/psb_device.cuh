@@ -171,6 +171,54 @@ __device__ __forceinline__ void node_bounds(const float *__restrict__ blk, const
     });
 }
 
+// S4 for the SS-tree variant (NEXT-2; §II-C, L499-504 §III):
+// child bounding spheres, block [d+1][F] = centroid rows then the radius row.
+// A sphere's MINDIST/MAXDIST need a square root, so unlike the MBR bounds they
+// cannot ride on monotone RN rounding; they are made safe explicitly:
+//   |q_j - c_j| rounded toward zero / away from zero, squares and sums rounded
+//   down / up, sqrt down / up, (sqrt - r) down, (sqrt + r) up, squared down / up,
+//   then scaled by (1 -/+ (2d+4) 2^-24), which covers the relative error of the
+//   RN point distance (recursive sum of d+2 rounded terms; R24).
+// So MINDIST <= dist_fl(q, p) <= MAXDIST for every point p inside the sphere,
+// which is all the exactness argument of §2 needs. Empty slots (centre +inf,
+// radius 0) give +inf for both.
+template <int D, int V, bool MAX>
+__device__ __forceinline__ void sphere_bounds(const float *__restrict__ blk, const Query<D> &q, int d, int lane,
+                                              float (&md)[V], float (&Md)[V])
+{
+    constexpr int F = 32 * V;
+    float lo2[V], hi2[V];
+#pragma unroll
+    for (int t = 0; t < V; ++t) { lo2[t] = 0.f; hi2[t] = 0.f; }
+    for_dims<D>(d, [&](int j) {
+        float c[V];
+        ldv<V>(blk + j * F + lane * V, c);
+        const float qj = q[j];
+#pragma unroll
+        for (int t = 0; t < V; ++t) {
+            const float a = fabsf(__fsub_rz(qj, c[t]));
+            lo2[t] = __fadd_rd(lo2[t], __fmul_rd(a, a));
+            if (MAX) {
+                const float b = fmaxf(__fsub_ru(qj, c[t]), __fsub_ru(c[t], qj));
+                hi2[t] = __fadd_ru(hi2[t], __fmul_ru(b, b));
+            }
+        }
+    });
+    float r[V];
+    ldv<V>(blk + d * F + lane * V, r);
+    const float g = __fmul_ru((float)(2 * d + 4), 5.9604644775390625e-8f);   // (2d+4) 2^-24
+    const float shrink = __fsub_rd(1.0f, g), grow = __fadd_ru(1.0f, g);
+#pragma unroll
+    for (int t = 0; t < V; ++t) {
+        const float dm = fmaxf(__fsub_rd(__fsqrt_rd(lo2[t]), r[t]), 0.0f);
+        md[t] = __fmul_rd(__fmul_rd(dm, dm), shrink);
+        if (MAX) {
+            const float dx = __fadd_ru(__fsqrt_ru(hi2[t]), r[t]);
+            Md[t] = __fmul_ru(__fmul_ru(dx, dx), grow);
+        }
+    }
+}
+
 // S8: distances of the query to this lane's V points of one leaf block [d][F].
 template <int D, int V>
 __device__ __forceinline__ void leaf_dists(const float *__restrict__ lp, const Query<D> &q, int d,

@@ -28,12 +28,15 @@ struct DevIndex {
     int32_t d;
     int32_t F;
     int32_t sm_count;                   // of the index's device (launch sizing)
+    int32_t sphere;                     // 0: MBR node blocks [d][2][F]; 1: sphere blocks [d+1][F]
+    int32_t blk_floats;                 // floats per internal node block
 };
 
 // Level geometry of a packed tree (shared by the host and GPU loaders).
 struct GpuLayoutShape {
     int64_t n = 0, L = 0;
     int32_t d = 0, F = 0, H = 0;
+    int32_t sphere = 0, blk_floats = 0;
     int64_t nlev[PSB_MAXLVL + 1] = {};
     int64_t level_off[PSB_MAXLVL + 1] = {};
     int64_t total_node_floats = 0;

@@ -22,12 +22,16 @@ int launch_tree(int algo, const DevIndex &ix, const float *queries, int64_t nq, 
 int launch_brute(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi, float *od,
                  cudaStream_t st, int sm_count, cudaMemPool_t pool);
 
-// Per-d launchers (instantiated in knn_tree_d*.cu / knn_brute_d*.cu); they
-// return PSB_NOT_INSTANTIATED when (d, fanout) needs the generic-d kernels.
+// Per-(d, fanout) launchers, instantiated one translation unit each
+// (knn_tree_d<D>_v<V>.cu, knn_brute_d<D>_v<V>.cu; V = fanout/32, D = 0: runtime d).
+// They return PSB_NOT_INSTANTIATED when the request needs the generic-d kernels.
 constexpr int PSB_NOT_INSTANTIATED = 1;
-template <int D>
-int launch_tree_v(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                  float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool, int parts);
+template <int D, int V>
+int launch_tree_ks(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
+                   float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool, int parts);
+template <int D, int V>
+int launch_brute_ks(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi, float *od,
+                    cudaStream_t st, int sm, cudaMemPool_t pool);
 
 // Latency-mode helpers (knn_merge.cu): shared pruning distances to +inf, and the
 // filtered merge of [nq][parts][k] per-part lists.
@@ -41,7 +45,7 @@ int launch_brute_v(const DevIndex &ix, const float *queries, int64_t nq, int k, 
 // GPU bulk load (psb_build_gpu.cu) into preallocated pts/ids/nodes; d_points is
 // device memory [n][d]. Synchronous on `st`.
 int gpu_bulk_load(const float *d_points, const GpuLayoutShape &sh, int64_t id_base, float *pts, int32_t *ids,
-                  float *nodes, cudaStream_t st);
+                  float *nodes, cudaStream_t st, bool sphere);
 
 // [parts][nq][k] sorted (dist, id) lists -> first k of their union (knn_brute.cu).
 int launch_merge(const int32_t *ids, const float *dists, int parts, int64_t nq, int k, int32_t *oi,

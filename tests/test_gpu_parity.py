@@ -173,13 +173,15 @@ def test_tie_heavy(kind):
     idx.free()
 
 
-def test_fma_case_on_gpu():
+@pytest.mark.parametrize("sphere", [False, True])
+def test_fma_case_on_gpu(sphere):
     import json, os
+    psb = _psb()
     g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "hand_cases.json")))["fma_case"]
     p = np.array([[float.fromhex(v) for v in g["point"]]] * 40, np.float32)
     q = np.array([[float.fromhex(v) for v in g["query"]]], np.float32)
-    idx = _psb().psb_build(p, 32)
-    for algo in ALGOS:
+    idx = psb.psb_build_ex(p, 32, packing=psb.PSB_NODE_SPHERE if sphere else 0)
+    for algo in (ALGOS if not sphere else ("psb", "bnb")):
         ids, d = run(idx, q, 1, algo)
         assert int(d.view(np.uint32)[0, 0]) == int(g["rn_bits"], 16)
     idx.free()
@@ -361,4 +363,63 @@ def test_split_edges(case):
     ids, d = psb.psb_knn_split(idx, torch.from_numpy(qs).cuda(), case["k"], parts=case["parts"])
     torch.cuda.synchronize()
     assert_same((ids.cpu().numpy(), d.cpu().numpy()), oracle.knn_bruteforce(pts, qs, case["k"]), str(case))
+    idx.free()
+
+
+@pytest.mark.parametrize("cfgname,nsub,nq", [("C1", None, 100), ("C2", 300_000, 2000), ("C3", 500_000, 300),
+                                             ("C4", 400_000, 100)])
+def test_sphere_index_parity(cfgname, nsub, nq):
+    """NEXT-2 SS-tree variant: sphere nodes (parallel Ritter, conservative radii,
+    directed-rounding bounds) give exactly the oracle's rows with PSB, B&B and
+    the latency mode."""
+    psb = _psb()
+    cfg = W.config(cfgname) if nsub is None else W.config(cfgname, n=nsub)
+    pts, qs = cfg.points(), cfg.queries(q=nq)
+    idx = psb.psb_build_ex(pts, cfg.fanout, packing=psb.PSB_NODE_SPHERE)
+    exp = oracle.Tree(pts).knn(qs, cfg.k)
+    for algo in ("psb", "bnb"):
+        for var in (0, 1):
+            assert_same(run(idx, qs, cfg.k, algo, var), exp, f"sphere {cfgname} {algo} var{var}")
+    ids, d = psb.psb_knn_split(idx, torch.from_numpy(qs[:8].copy()).cuda(), cfg.k, parts=32)
+    torch.cuda.synchronize()
+    assert_same((ids.cpu().numpy(), d.cpu().numpy()), (exp[0][:8], exp[1][:8]), "sphere split")
+    idx.free()
+
+
+@pytest.mark.parametrize("case", [dict(n=1, d=2, F=32), dict(n=5_000, d=1, F=32), dict(n=20_000, d=64, F=64),
+                                  dict(n=33_333, d=7, F=256), dict(n=10_000, d=3, F=32, dups=True)])
+def test_sphere_containment_and_parity(case):
+    """Every point lies inside its leaf's sphere and every child sphere inside its
+    parent's, checked in float64 on the exported index; and results are exact."""
+    psb = _psb()
+    rng = np.random.default_rng(case["n"] + case["d"])
+    if case.get("dups"):
+        pts = rng.integers(0, 4, size=(case["n"], case["d"])).astype(np.float32)
+    else:
+        pts = (rng.normal(size=(case["n"], case["d"])) * 20).astype(np.float32)
+    idx = psb.psb_build_ex(pts, case["F"], packing=psb.PSB_NODE_SPHERE)
+    ex = psb.psb_index_export(idx)
+    assert ex["sphere"]
+    F, d, L = ex["fanout"], ex["d"], ex["leaves"]
+    lv1 = ex["nodes"][1]
+    for j in range(L):
+        c = lv1[j // F, :d, j % F].astype(np.float64)
+        r = float(lv1[j // F, d, j % F])
+        cnt = min(F, ex["n"] - j * F)
+        P = ex["pts"][j, :, :cnt].T.astype(np.float64)
+        assert (np.sqrt(((P - c) ** 2).sum(1)) <= r).all()
+    for lv in range(2, ex["levels"] + 1):
+        below, cur = ex["nodes"][lv - 1], ex["nodes"][lv]
+        for g in range(below.shape[0]):
+            pc = cur[g // F, :d, g % F].astype(np.float64)
+            pr = float(cur[g // F, d, g % F])
+            cnt = min(F, ex["nlev"][lv - 2] - g * F)
+            cc = below[g, :d, :cnt].T.astype(np.float64)
+            cr = below[g, d, :cnt].astype(np.float64)
+            assert (np.sqrt(((cc - pc) ** 2).sum(1)) + cr <= pr * (1 + 1e-6) + 1e-6).all()
+    qs = (rng.normal(size=(40, case["d"])) * 25).astype(np.float32)
+    for k in (1, 17, 64):
+        exp = oracle.knn_bruteforce(pts, qs, k)
+        for algo in ("psb", "bnb"):
+            assert_same(run(idx, qs, k, algo), exp, f"{case} k={k} {algo}")
     idx.free()
