@@ -71,7 +71,8 @@ enum { PSB_PACK_HILBERT = 0, PSB_PACK_STR = 1 };
  * loader only (not with PSB_BUILD_HOST / PSB_PACK_STR). */
 #define PSB_NODE_SPHERE 0x200u
 
-#define PSB_KMAX 128          /* largest k served by the warp top-k (4 keys per lane) */
+#define PSB_KMAX 2048         /* largest k: <= 128 in registers (4 keys per lane), up to
+                                 2048 in a per-warp shared-memory list (NEXT-3) */
 #define PSB_DMAX 64           /* largest dimensionality                               */
 
 /* Bulk-load an R-tree over points[n][d] (§IV, bottom-up construction,
@@ -104,7 +105,9 @@ int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int6
  * the leftmost child within the pruning distance whose leaves are not yet
  * visited (l.16-26), scans leaves left to right while they improve the kNN set
  * (l.32-41) and backtracks through parent links otherwise (l.27-30, l.42-45).
- * 1 <= k <= PSB_KMAX (else PSB_EUNSUPPORTED), q >= 0 (q = 0 is a no-op). */
+ * 1 <= k <= PSB_KMAX (else PSB_EUNSUPPORTED), q >= 0 (q = 0 is a no-op).
+ * For k > 128 the kNN list lives in shared memory (§V-E future
+ * work: large k) and psb_knn_split runs as psb_knn. */
 int psb_knn(const psb_index *idx, const float *queries, int64_t q, int32_t k,
             int32_t *out_ids, float *out_dists, void *stream);
 

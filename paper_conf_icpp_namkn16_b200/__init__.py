@@ -27,7 +27,7 @@ PSB_BUILD_HOST = 0x100
 PSB_NODE_SPHERE = 0x200
 PSB_ALGO_PSB, PSB_ALGO_BNB, PSB_ALGO_BRUTE = 0, 1, 2
 PSB_VAR_NOCACHE, PSB_VAR_NOMAXDIST = 1, 2
-PSB_KMAX, PSB_DMAX = 128, 64
+PSB_KMAX, PSB_DMAX = 2048, 64
 FANOUTS = (32, 64, 128, 256, 512)
 
 # every symbol include/psb.h declares (tests check the .so exports all of them)

@@ -29,8 +29,11 @@ brute_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k, 
     const int64_t q0 = ((int64_t)blockIdx.x * BF_WARPS + w) * QW;
     if (q0 >= nq) return;
     const int d = ix.d;
-    u64 *scratch = reinterpret_cast<u64 *>(smem) + (size_t)w * 32;
-    float *qs = reinterpret_cast<float *>(smem + BF_WARPS * 32 * 8) + (size_t)w * QW * PSB_DMAX;
+    // per warp: 32-key merge scratch, then (large k) QW lists of k keys; queries after all warps
+    const size_t per_warp = 32 + (KS == 0 ? (size_t)QW * k : 0);
+    u64 *scratch = reinterpret_cast<u64 *>(smem) + (size_t)w * per_warp;
+    u64 *lists = scratch + 32;
+    float *qs = reinterpret_cast<float *>(smem + BF_WARPS * per_warp * 8) + (size_t)w * QW * PSB_DMAX;
 
     Query<D> q[QW];
 #pragma unroll
@@ -41,7 +44,7 @@ brute_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k, 
     TopK<KS> T[QW];
     u64 thr[QW];
 #pragma unroll
-    for (int i = 0; i < QW; ++i) { T[i].init(); thr[i] = PAD_KEY; }
+    for (int i = 0; i < QW; ++i) { T[i].init(lists + (size_t)i * k, k); thr[i] = PAD_KEY; }
 
     const int64_t l0 = (int64_t)blockIdx.y * leaves_per_chunk;
     const int64_t l1 = l0 + leaves_per_chunk < ix.L ? l0 + leaves_per_chunk : ix.L;
@@ -84,7 +87,7 @@ template <int D, int V, int KS>
 static int launch_brute_t(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
                           float *od, cudaStream_t st, int sm_count, cudaMemPool_t pool)
 {
-    constexpr int QW = KS >= 4 ? 2 : 4;
+    constexpr int QW = KS == 0 ? 1 : (KS >= 4 ? 2 : 4);
     const int64_t warps_q = (nq + QW - 1) / QW;
     const int64_t blocks_q = (warps_q + BF_WARPS - 1) / BF_WARPS;
     // enough warps to cover ~48 per SM; chunks never smaller than 4 leaves
@@ -95,7 +98,13 @@ static int launch_brute_t(const DevIndex &ix, const float *queries, int64_t nq, 
     if (S < 1) S = 1;
     const int64_t per = (ix.L + S - 1) / S;
     S = (ix.L + per - 1) / per;
-    const size_t smem = BF_WARPS * 32 * 8 + (D == 0 ? (size_t)BF_WARPS * QW * PSB_DMAX * 4 : 0);
+    const size_t smem = BF_WARPS * (32 + (KS == 0 ? (size_t)QW * k : 0)) * 8 +
+                        (D == 0 ? (size_t)BF_WARPS * QW * PSB_DMAX * 4 : 0);
+    if (smem > 48 * 1024) {
+        cudaError_t ea = cudaFuncSetAttribute(brute_kernel<D, V, KS, QW>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                              (int)smem);
+        if (ea != cudaSuccess) return report_cuda(ea, "cudaFuncSetAttribute (brute)");
+    }
     int32_t *pi = oi;
     float *pd = od;
     if (S > 1) {
@@ -121,7 +130,10 @@ int launch_brute_ks(const DevIndex &ix, const float *queries, int64_t nq, int k,
 {
     if (k <= 32) return launch_brute_t<D, V, 1>(ix, queries, nq, k, oi, od, st, sm, pool);
     if (k <= 64) return launch_brute_t<D, V, 2>(ix, queries, nq, k, oi, od, st, sm, pool);
-    if constexpr (D == 0) return launch_brute_t<D, V, 4>(ix, queries, nq, k, oi, od, st, sm, pool);
+    if constexpr (D == 0) {
+        if (k <= 128) return launch_brute_t<D, V, 4>(ix, queries, nq, k, oi, od, st, sm, pool);
+        return launch_brute_t<D, V, 0>(ix, queries, nq, k, oi, od, st, sm, pool);   // NEXT-3
+    }
     return PSB_NOT_INSTANTIATED;   // k > 64: generic-d kernels
 }
 

@@ -13,27 +13,27 @@ __global__ void __launch_bounds__(128)
 merge_kernel(const int32_t *__restrict__ ids, const float *__restrict__ dists, int parts, int64_t nq,
              int k, int32_t *__restrict__ out_ids, float *__restrict__ out_dists)
 {
-    __shared__ u64 scratch_all[4 * 32];
-    u64 *scratch = scratch_all + (threadIdx.x >> 5) * 32;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const size_t per_warp = 32 + (KS == 0 ? (size_t)k : 0);
+    u64 *scratch = reinterpret_cast<u64 *>(smem_raw) + (threadIdx.x >> 5) * per_warp;
     const int lane = threadIdx.x & 31;
     const int64_t qi = (int64_t)blockIdx.x * 4 + (threadIdx.x >> 5);
     if (qi >= nq) return;
     TopK<KS> T;
-#pragma unroll
-    for (int s = 0; s < KS; ++s) {
-        const int r = s * 32 + lane;
-        T.key[s] = r < k ? make_key(__ldg(dists + qi * k + r), __ldg(ids + qi * k + r)) : PAD_KEY;
-    }
-    u64 thr = T.kth(k);
-    for (int p = 1; p < parts; ++p) {
+    T.init(scratch + 32, k);
+    u64 thr = PAD_KEY;
+    constexpr int C = KS == 0 ? 4 : KS;      // keys per lane per offer round
+    for (int p = 0; p < parts; ++p) {
         const int64_t row = ((int64_t)p * nq + qi) * k;
-        u64 cand[KS];
+        for (int r0 = 0; r0 < k; r0 += 32 * C) {
+            u64 cand[C];
 #pragma unroll
-        for (int s = 0; s < KS; ++s) {
-            const int r = s * 32 + lane;
-            cand[s] = r < k ? make_key(__ldg(dists + row + r), __ldg(ids + row + r)) : ~0ull;
+            for (int s = 0; s < C; ++s) {
+                const int r = r0 + s * 32 + lane;
+                cand[s] = r < k ? make_key(__ldg(dists + row + r), __ldg(ids + row + r)) : ~0ull;
+            }
+            T.template offer<C>(cand, k, lane, thr, scratch);
         }
-        T.template offer<KS>(cand, k, lane, thr, scratch);
     }
     T.store(k, lane, out_ids + qi * k, out_dists + qi * k);
 }
@@ -121,9 +121,18 @@ int launch_merge(const int32_t *ids, const float *dists, int parts, int64_t nq, 
                  float *od, cudaStream_t st)
 {
     const unsigned blocks = (unsigned)((nq + 3) / 4);
-    if (k <= 32) merge_kernel<1><<<blocks, 128, 0, st>>>(ids, dists, parts, nq, k, oi, od);
-    else if (k <= 64) merge_kernel<2><<<blocks, 128, 0, st>>>(ids, dists, parts, nq, k, oi, od);
-    else merge_kernel<4><<<blocks, 128, 0, st>>>(ids, dists, parts, nq, k, oi, od);
+    const size_t s0 = 4 * 32 * 8;
+    if (k <= 32) merge_kernel<1><<<blocks, 128, s0, st>>>(ids, dists, parts, nq, k, oi, od);
+    else if (k <= 64) merge_kernel<2><<<blocks, 128, s0, st>>>(ids, dists, parts, nq, k, oi, od);
+    else if (k <= 128) merge_kernel<4><<<blocks, 128, s0, st>>>(ids, dists, parts, nq, k, oi, od);
+    else {
+        const size_t sb = 4 * (32 + (size_t)k) * 8;         // NEXT-3: list in shared memory
+        if (sb > 48 * 1024) {
+            cudaError_t ea = cudaFuncSetAttribute(merge_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sb);
+            if (ea != cudaSuccess) return report_cuda(ea, "cudaFuncSetAttribute (merge)");
+        }
+        merge_kernel<0><<<blocks, 128, sb, st>>>(ids, dists, parts, nq, k, oi, od);
+    }
     return report_cuda(cudaGetLastError(), "merge kernel launch");
 }
 

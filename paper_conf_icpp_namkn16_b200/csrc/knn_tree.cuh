@@ -21,13 +21,14 @@ struct WarpState {
     float *cache_md;     // [(H+1)][F] child MINDISTs of the node cached per level
     int32_t *cache_node; // [(H+1)] node id cached per level (-1 = none)
     u64 *scratch;        // [32] top-k merge scratch
+    u64 *list;           // [k] large-k list (KS == 0 kernels)
     float *qsmem;        // query (D == 0 only)
 };
 
-__device__ __forceinline__ WarpState warp_state(unsigned char *smem, int H, int F, bool qsmem)
+__device__ __forceinline__ WarpState warp_state(unsigned char *smem, int H, int F, bool qsmem, int kbig = 0)
 {
     const int w = threadIdx.x >> 5;
-    unsigned char *base = smem + (size_t)w * WarpSmem::bytes(H, F, qsmem);
+    unsigned char *base = smem + (size_t)w * WarpSmem::bytes(H, F, qsmem, kbig);
     WarpState s;
     s.cache_md = reinterpret_cast<float *>(base);
     size_t off = (WarpSmem::cache_floats(H, F) * 4 + 15) & ~(size_t)15;
@@ -36,6 +37,8 @@ __device__ __forceinline__ WarpState warp_state(unsigned char *smem, int H, int 
     off = (off + 15) & ~(size_t)15;
     s.scratch = reinterpret_cast<u64 *>(base + off);
     off += 32 * 8;
+    s.list = reinterpret_cast<u64 *>(base + off);
+    off += (size_t)kbig * 8;
     s.qsmem = reinterpret_cast<float *>(base + off);
     return s;
 }
@@ -107,7 +110,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     for (int l = lane; l <= H; l += 32) ws.cache_node[l] = -1;
     __syncwarp();
     TopK<KS> T;
-    T.init();
+    T.init(ws.list, k);
     u64 thr = PAD_KEY;
     float pd = __int_as_float(0x7f800000);
     Stats<ST> S;
@@ -223,7 +226,7 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
     for (int l = lane; l <= H; l += 32) ws.cache_node[l] = -1;
     __syncwarp();
     TopK<KS> T;
-    T.init();
+    T.init(ws.list, k);
     u64 thr = PAD_KEY;
     float pd = __int_as_float(0x7f800000);
     Stats<ST> S;
@@ -288,7 +291,7 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
     {                                                                                                 \
         extern __shared__ __align__(16) unsigned char smem[];                                         \
         const int lane = threadIdx.x & 31;                                                            \
-        const WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0);                                  \
+        const WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);                 \
         const bool use_cache = !(variant & PSB_VAR_NOCACHE);                                          \
         const bool use_max = !(variant & PSB_VAR_NOMAXDIST);                                          \
         int64_t qi = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);                        \
@@ -339,7 +342,7 @@ __device__ __forceinline__ void psb_part_query(const DevIndex &ix, const float *
     const int chunk = (L + parts - 1) / parts;
     const int lo = part * chunk, hi = min(lo + chunk, L);
     TopK<KS> T;
-    T.init();
+    T.init(ws.list, k);
     int32_t *oi = part_ids + (qi * parts + part) * (int64_t)k;
     float *od = part_dists + (qi * parts + part) * (int64_t)k;
     if (lo >= hi) {
@@ -453,7 +456,7 @@ psb_split_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int
     const int lane = threadIdx.x & 31;
     const int64_t w = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
     if (w >= nq * parts) return;
-    const WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0);
+    const WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);
     psb_part_query<D, V, KS, ST, SPH>(ix, queries, w / parts, (int)(w % parts), parts, k, part_ids, part_dists, gpd, ws,
                                  !(variant & PSB_VAR_NOCACHE), !(variant & PSB_VAR_NOMAXDIST), lane);
 }
@@ -463,7 +466,7 @@ static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int
                          int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats,
                          cudaMemPool_t pool, int parts)
 {
-    const size_t smem = WARPS_PER_CTA * WarpSmem::bytes(ix.H, 32 * V, D == 0);
+    const size_t smem = WARPS_PER_CTA * WarpSmem::bytes(ix.H, 32 * V, D == 0, KS == 0 ? k : 0);
     int64_t blocks = (nq + WARPS_PER_CTA - 1) / WARPS_PER_CTA;
     // Counting (stats) kernels are instantiated for the generic-d path only: the
     // traversal, hence every counter, does not depend on the d specialisation.
@@ -488,7 +491,7 @@ static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int
         e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return report_cuda(e, "cudaFuncSetAttribute");
     }
-    if (parts > 1 && algo == PSB_ALGO_PSB && !stats) {
+    if (parts > 1 && algo == PSB_ALGO_PSB && !stats && KS != 0) {
         // latency mode: q*parts warps, shared pd per query, then a filtered merge
         auto sk = ix.sphere ? psb_split_kernel<D, V, KS, false, true> : psb_split_kernel<D, V, KS, false, false>;
         if (smem > 48 * 1024) {
@@ -543,7 +546,10 @@ int launch_tree_ks(int algo, const DevIndex &ix, const float *queries, int64_t n
 {
     if (k <= 32) return launch_tree_t<D, V, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
     if (k <= 64) return launch_tree_t<D, V, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
-    if constexpr (D == 0) return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
+    if constexpr (D == 0) {
+        if (k <= 128) return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
+        return launch_tree_t<D, V, 0>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);  // NEXT-3
+    }
     return PSB_NOT_INSTANTIATED;   // k > 64: generic-d kernels (keeps compile time down)
 }
 

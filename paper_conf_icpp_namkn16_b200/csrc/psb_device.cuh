@@ -310,6 +310,7 @@ struct TopK {
 #pragma unroll
         for (int s = 0; s < KS; ++s) key[s] = PAD_KEY;
     }
+    __device__ __forceinline__ void init(u64 *, int) { init(); }
     // key at position k-1 (the current k-th neighbour), warp-uniform
     __device__ __forceinline__ u64 kth(int k) const
     {
@@ -456,6 +457,83 @@ struct Stats {
     }
 };
 
+
+// NEXT-3 (large k, §V-E: "the kNN list grows with k
+// ... future work: store large distances in shared memory"): for k > 128 the
+// sorted list lives in per-warp shared memory (k u64 keys) instead of registers.
+// Candidates below the k-th key are compacted (<= 32 per round), bitonic-sorted,
+// and merged in place: list keys at positions >= the first insertion point move
+// right by the number of candidates below them (processed in 32-key chunks from
+// the end, so every key is read before its slot is overwritten) and candidates
+// drop into the gaps; positions >= k fall off.
+template <>
+struct TopK<0> {
+    u64 *list;   // [k] ascending, shared memory
+
+    __device__ __forceinline__ void init(u64 *smem_list, int k)
+    {
+        list = smem_list;
+        for (int i = threadIdx.x & 31; i < k; i += 32) list[i] = PAD_KEY;
+        __syncwarp();
+    }
+    __device__ __forceinline__ u64 kth(int k) const { return list[k - 1]; }
+
+    // number of keys < x in the ascending a[0..n)
+    static __device__ __forceinline__ int rank(const u64 *a, int n, u64 x)
+    {
+        int lo = 0, hi = n;
+        while (lo < hi) {
+            const int mid = (lo + hi) >> 1;
+            if (a[mid] < x) lo = mid + 1;
+            else hi = mid;
+        }
+        return lo;
+    }
+
+    template <int V>
+    __device__ __forceinline__ int offer(const u64 (&cand)[V], int k, int lane, u64 &thr, u64 *scratch)
+    {
+        int total = 0;
+        const unsigned lt = (1u << lane) - 1;
+#pragma unroll
+        for (int t = 0; t < V; ++t) {
+            const unsigned b = __ballot_sync(FULL, cand[t] < thr);
+            const int m = __popc(b);
+            if (m == 0) continue;
+            total += m;
+            if (b >> lane & 1u) scratch[__popc(b & lt)] = cand[t];
+            __syncwarp();
+            u64 c = lane < m ? scratch[lane] : ~0ull;
+            __syncwarp();
+            c = m <= 8 ? warp_sort32<8>(c, lane) : (m <= 16 ? warp_sort32<16>(c, lane) : warp_sort32<32>(c, lane));
+            scratch[lane] = c;
+            __syncwarp();
+            const int rc = lane < m ? rank(list, k, c) : k;       // candidate's rank among the old keys
+            const int p0 = __shfl_sync(FULL, rc, 0);               // first insertion point
+            for (int base = ((k - 1) >> 5) << 5; base >= 0 && base + 31 >= p0; base -= 32) {
+                const int i = base + lane;
+                const bool mv = i < k && i >= p0;
+                const u64 a = mv ? list[i] : 0ull;
+                const int sh = mv ? rank(scratch, m, a) : 0;
+                __syncwarp();
+                if (mv && i + sh < k) list[i + sh] = a;
+                __syncwarp();
+            }
+            if (lane < m && lane + rc < k) list[lane + rc] = c;
+            __syncwarp();
+            thr = list[k - 1];
+        }
+        return total;
+    }
+    __device__ __forceinline__ void store(int k, int lane, int32_t *__restrict__ oi, float *__restrict__ od) const
+    {
+        for (int r = lane; r < k; r += 32) {
+            oi[r] = key_id(list[r]);
+            od[r] = key_dist(list[r]);
+        }
+    }
+};
+
 // S8+S9: scan one leaf, offer its points. Ids are fetched lazily, only for
 // points whose distance can enter the list (dist <= current k-th distance).
 template <int D, int V, int KS, bool ST>
@@ -489,13 +567,14 @@ __device__ __forceinline__ bool scan_leaf(const DevIndex &ix, int leaf, const Qu
 // Per-warp shared-memory layout for the traversal kernels.
 struct WarpSmem {
     static __host__ __device__ __forceinline__ size_t cache_floats(int H, int F) { return (size_t)(H + 1) * F; }
-    static __host__ __device__ __forceinline__ size_t bytes(int H, int F, bool qsmem)
+    static __host__ __device__ __forceinline__ size_t bytes(int H, int F, bool qsmem, int kbig = 0)
     {
         size_t b = cache_floats(H, F) * 4;
         b = (b + 15) & ~(size_t)15;
         b += (size_t)(H + 1) * 4;
         b = (b + 15) & ~(size_t)15;
         b += 32 * 8;                        // top-k merge scratch
+        b += (size_t)kbig * 8;              // large-k list (TopK<0>)
         if (qsmem) b += PSB_DMAX * 4;
         return b;
     }

@@ -38,7 +38,8 @@ def test_argument_errors_without_gpu():
     assert "NULL" in psb.psb_last_error()
     assert L.psb_knn_ex(None, None, 1, 8, None, None, None, 0, 0) == psb.PSB_EINVAL
     assert L.psb_merge_topk(None, None, 0, 1, 8, None, None, None) == psb.PSB_EINVAL
-    assert L.psb_merge_topk(None, None, 2, 1, 200, None, None, None) == psb.PSB_EUNSUPPORTED
+    assert L.psb_merge_topk(None, None, 2, 1, psb.PSB_KMAX + 1, None, None, None) == psb.PSB_EUNSUPPORTED
+    assert L.psb_merge_topk(None, None, 2, 1, 200, None, None, None) == psb.PSB_EINVAL   # NULL buffers
     assert L.psb_index_info(None, None, None, None, None, None, None) == psb.PSB_EINVAL
     out = ctypes.c_void_p()
     assert L.psb_build_ex(None, 10, 2, 32, 0, 0, ctypes.byref(out)) == psb.PSB_EINVAL

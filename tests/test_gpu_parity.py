@@ -262,7 +262,7 @@ def test_error_codes_on_gpu():
         psb.psb_knn(idx, qd, 0)
     assert e.value.code == psb.PSB_EINVAL
     with pytest.raises(psb.PSBError) as e:
-        psb.psb_knn(idx, qd, 129)
+        psb.psb_knn(idx, qd, psb.PSB_KMAX + 1)
     assert e.value.code == psb.PSB_EUNSUPPORTED
     # q = 0 is a no-op
     ids, d = psb.psb_knn(idx, torch.zeros((0, 2), device="cuda"), 5)
@@ -422,4 +422,44 @@ def test_sphere_containment_and_parity(case):
         exp = oracle.knn_bruteforce(pts, qs, k)
         for algo in ("psb", "bnb"):
             assert_same(run(idx, qs, k, algo), exp, f"{case} k={k} {algo}")
+    idx.free()
+
+
+@pytest.mark.parametrize("k", [129, 200, 512, 1000, 2048])
+def test_large_k(c2, k):
+    """NEXT-3: k > 128 (shared-memory kNN list, in-place merge insertion) for
+    PSB, B&B, brute force (with its chunk merge) and the split entry point."""
+    psb = _psb()
+    cfg, pts, qs, idx, _ = c2
+    sub = qs[:40]
+    exp = oracle.Tree(pts).knn(sub, k)
+    for algo in ALGOS:
+        assert_same(run(idx, sub, k, algo), exp, f"k={k} {algo}")
+    ids, d = psb.psb_knn_split(idx, torch.from_numpy(sub[:4].copy()).cuda(), k)
+    torch.cuda.synchronize()
+    assert_same((ids.cpu().numpy(), d.cpu().numpy()), (exp[0][:4], exp[1][:4]), f"k={k} split")
+
+
+def test_large_k_small_n_and_merge():
+    psb = _psb()
+    rng = np.random.default_rng(8)
+    pts = rng.integers(0, 7, size=(700, 3)).astype(np.float32)    # ties everywhere, k > n
+    qs = rng.integers(0, 7, size=(20, 3)).astype(np.float32)
+    idx = psb.psb_build(pts, 32)
+    exp = oracle.knn_bruteforce(pts, qs, 1000)
+    for algo in ALGOS:
+        assert_same(run(idx, qs, 1000, algo), exp, f"k>n {algo}")
+    # data-sharded merge with large k
+    b = [0, 250, 700]
+    ids = torch.empty((2, 20, 300), dtype=torch.int32, device="cuda")
+    ds = torch.empty((2, 20, 300), dtype=torch.float32, device="cuda")
+    for r in range(2):
+        sub = psb.psb_build_ex(pts[b[r]:b[r + 1]], 32, id_base=b[r])
+        psb.psb_knn(sub, torch.from_numpy(qs).cuda(), 300, out=(ids[r], ds[r]))
+        torch.cuda.synchronize()
+        sub.free()
+    mi, md = psb.psb_merge_topk(ids, ds, 300)
+    torch.cuda.synchronize()
+    e = oracle.knn_bruteforce(pts, qs, 300)
+    assert_same((mi.cpu().numpy(), md.cpu().numpy()), e, "merge k=300")
     idx.free()
