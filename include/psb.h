@@ -56,7 +56,12 @@ enum {
 
 /* Leaf packing order for psb_build_ex `flags` (§IV-A: sort points by
  * a space-filling-curve key and pack them into full leaves, bottom-up). */
-enum { PSB_PACK_HILBERT = 0, PSB_PACK_STR = 1 };
+enum { PSB_PACK_HILBERT = 0, PSB_PACK_STR = 1, PSB_PACK_KMEANS = 2 };
+/* PSB_PACK_KMEANS (NEXT-4, §IV-B): k-means with k = number of leaves
+ * (P:L586-587), initialised from the Hilbert leaves, 4 Lloyd iterations whose
+ * assignment step is this library's own exact 1-NN search over the centroids;
+ * leaves are then packed cluster by cluster in the Hilbert order of the
+ * centroids. GPU loader only. Deterministic. */
 /* Build-location flag (OR into psb_build_ex `flags`). Hilbert packing runs on
  * the GPU by default (keys, CUB radix sort, permutation and MBR levels in CUDA
  * kernels; NEXT-1); PSB_BUILD_HOST forces the host (OpenMP) loader. STR always

@@ -22,7 +22,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("PSB_LIB_PATH") or os.path.join(_HERE, "libpsb.so")   # override: A/B builds
 
 PSB_OK, PSB_EINVAL, PSB_ENOMEM, PSB_ECUDA, PSB_EUNSUPPORTED = 0, -1, -2, -3, -4
-PSB_PACK_HILBERT, PSB_PACK_STR = 0, 1
+PSB_PACK_HILBERT, PSB_PACK_STR, PSB_PACK_KMEANS = 0, 1, 2
 PSB_BUILD_HOST = 0x100
 PSB_NODE_SPHERE = 0x200
 PSB_ALGO_PSB, PSB_ALGO_BNB, PSB_ALGO_BRUTE = 0, 1, 2

@@ -116,10 +116,11 @@ int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int6
     int rc = psb_layout_shape(n, d, fanout, id_base, flags, &shape);
     if (rc != PSB_OK) return rc;
     const bool sphere = (flags & PSB_NODE_SPHERE) != 0;
-    const bool on_gpu = (flags & ~(uint32_t)(PSB_BUILD_HOST | PSB_NODE_SPHERE)) == PSB_PACK_HILBERT &&
-                        !(flags & PSB_BUILD_HOST);
-    if (sphere && !on_gpu) {
-        psb_set_error("psb_build_ex: PSB_NODE_SPHERE needs the GPU Hilbert loader");
+    const uint32_t pack = flags & ~(uint32_t)(PSB_BUILD_HOST | PSB_NODE_SPHERE);
+    const bool kmeans = pack == PSB_PACK_KMEANS;
+    const bool on_gpu = (pack == PSB_PACK_HILBERT || kmeans) && !(flags & PSB_BUILD_HOST);
+    if ((sphere || kmeans) && !on_gpu) {
+        psb_set_error("psb_build_ex: PSB_NODE_SPHERE / PSB_PACK_KMEANS need the GPU loader");
         return PSB_EUNSUPPORTED;
     }
     cudaPointerAttributes attr;
@@ -172,7 +173,7 @@ int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int6
             }
             dpts = staged;
         }
-        rc = psb::gpu_bulk_load(dpts, shape, id_base, ix->pts, ix->ids, ix->nodes, st, sphere);
+        rc = psb::gpu_bulk_load(dpts, shape, id_base, ix->pts, ix->ids, ix->nodes, st, sphere, kmeans ? 4 : 0);
         cudaStreamSynchronize(st);
         cudaFree(staged);
         cudaStreamDestroy(st);

@@ -45,7 +45,7 @@ int launch_brute_v(const DevIndex &ix, const float *queries, int64_t nq, int k, 
 // GPU bulk load (psb_build_gpu.cu) into preallocated pts/ids/nodes; d_points is
 // device memory [n][d]. Synchronous on `st`.
 int gpu_bulk_load(const float *d_points, const GpuLayoutShape &sh, int64_t id_base, float *pts, int32_t *ids,
-                  float *nodes, cudaStream_t st, bool sphere);
+                  float *nodes, cudaStream_t st, bool sphere, int kmeans_iters);
 
 // [parts][nq][k] sorted (dist, id) lists -> first k of their union (knn_brute.cu).
 int launch_merge(const int32_t *ids, const float *dists, int parts, int64_t nq, int k, int32_t *oi,

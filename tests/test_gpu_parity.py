@@ -463,3 +463,25 @@ def test_large_k_small_n_and_merge():
     e = oracle.knn_bruteforce(pts, qs, 300)
     assert_same((mi.cpu().numpy(), md.cpu().numpy()), e, "merge k=300")
     idx.free()
+
+
+@pytest.mark.parametrize("sphere", [False, True])
+def test_kmeans_packing_parity(sphere):
+    """NEXT-4 k-means packing (k = #leaves, Lloyd steps via the library's own exact
+    1-NN): a valid packing (every point exactly once) and exact results."""
+    psb = _psb()
+    cfg = W.config("C2", n=200_000)
+    pts, qs = cfg.points(), cfg.queries(q=1000)
+    flags = psb.PSB_PACK_KMEANS | (psb.PSB_NODE_SPHERE if sphere else 0)
+    idx = psb.psb_build_ex(pts, cfg.fanout, packing=flags)
+    ex = psb.psb_index_export(idx)
+    ids = ex["ids"].reshape(-1)
+    assert sorted(ids[ids >= 0].tolist()) == list(range(len(pts)))
+    exp = oracle.Tree(pts).knn(qs, cfg.k)
+    for algo in ("psb", "bnb"):
+        assert_same(run(idx, qs, cfg.k, algo), exp, f"kmeans sphere={sphere} {algo}")
+    # deterministic
+    idx2 = psb.psb_build_ex(pts, cfg.fanout, packing=flags)
+    assert np.array_equal(psb.psb_index_export(idx2)["ids"], ex["ids"])
+    idx.free()
+    idx2.free()
