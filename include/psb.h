@@ -145,9 +145,18 @@ int psb_knn_bruteforce(const psb_index *idx, const float *queries, int64_t q, in
  * bit 0 PSB_VAR_NOCACHE  — re-fetch every node on return instead of reusing the
  *                          per-level MINDIST path cache (the paper's parent-link
  *                          behaviour);
- * bit 1 PSB_VAR_NOMAXDIST — skip the k-th-MAXDIST bound (Alg. 1 l.13-15).
+ * bit 1 PSB_VAR_NOMAXDIST — skip the k-th-MAXDIST bound (Alg. 1 l.13-15);
+ * bit 2 PSB_VAR_INPUT_ORDER — process the queries in input order;
+ * bit 3 PSB_VAR_LEAF_ORDER — process them in the order of their ClosestLeaf: the
+ *                          batch is first sorted (stably) by the sequence id of
+ *                          the leaf PSB's pass 1 descends to (Alg. 1 l.3),
+ *                          so warps running together walk neighbouring leaves and
+ *                          share them in L1/L2. Rows are still written in input
+ *                          order. With neither bit, leaf order is used when
+ *                          q >= 1024 and the leaves (points + ids) exceed 64 MiB.
  * Results are identical for every variant. */
-enum { PSB_VAR_NOCACHE = 1, PSB_VAR_NOMAXDIST = 2 };
+enum { PSB_VAR_NOCACHE = 1, PSB_VAR_NOMAXDIST = 2, PSB_VAR_INPUT_ORDER = 4,
+       PSB_VAR_LEAF_ORDER = 8 };
 int psb_knn_ex(const psb_index *idx, const float *queries, int64_t q, int32_t k,
                int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant);
 enum { PSB_ALGO_PSB = 0, PSB_ALGO_BNB = 1, PSB_ALGO_BRUTE = 2 };

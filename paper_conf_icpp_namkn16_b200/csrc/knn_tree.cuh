@@ -13,6 +13,11 @@
 namespace psb {
 
 constexpr int WARPS_PER_CTA = 4;
+// Batches are reordered by closest leaf (knn_order.cu) by default when they have
+// at least this many queries and the leaves (points + ids) do not sit in L2
+// anyway (profiles/r01_query_order.md: a loss at C2's 16 MB, a gain from C3's 146 MB).
+constexpr int64_t REORDER_MIN_QUERIES = 1024;
+constexpr double REORDER_MIN_BYTES = 64.0 * (1 << 20);
 #ifndef PSB_MIN_BLOCKS
 #define PSB_MIN_BLOCKS 8   // <= 64 registers: measured best on C2/C3 (profiles/r01_occupancy.md)
 #endif
@@ -115,69 +120,66 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     float pd = __int_as_float(0x7f800000);
     Stats<ST> S;
 
+    // One loop runs both passes so that each step (node bounds, leaf scan, top-k
+    // merge) is inlined once: the kernel's code size decides its instruction-cache
+    // hit rate (profiles/r01_icache.md).
+    //
     // S2: pass 1, getInitialPruningDistance(Q, ClosestLeaf) (Alg. 1 l.3; R4):
-    // greedy descent by (MINDIST, child index) argmin, k-th-MAXDIST bounds on the way.
-    int lvl = H;
-    int node = 0;
-    while (lvl > 0) {
-        float md[V];
-        S.node(internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
-        const int base = node * F, nb = (int)ix.nlev[lvl - 1];
-        u64 best = ~0ull;
-#pragma unroll
-        for (int t = 0; t < V; ++t) {
-            const int c = lane * V + t;
-            if (base + c < nb) {
-                const u64 kk = make_key(md[t], c);
-                best = kk < best ? kk : best;
-            }
-        }
-        best = warp_min_u64(best);
-        node = base + (int)(best & 0xffffffffu);
-        --lvl;
-    }
-    // ClosestLeaf and its right siblings until k points are seen; their points go
-    // straight into the kNN list (allowed by R4: pass 2 then skips these leaves).
-    const int pass1_lo = node;
-    int pass1_hi = node - 1;
-    int64_t seen = 0;
-    while (seen < k && pass1_hi + 1 < (int)ix.L) {
-        ++pass1_hi;
-        scan_leaf<D, V, KS, ST>(ix, pass1_hi, q, lane, T, k, thr, S, ws.scratch);
-        const int64_t left = ix.n - (int64_t)pass1_hi * F;
-        seen += left < F ? left : F;
-    }
-    pd = fminf(pd, key_dist(thr));
-
+    // greedy descent by (MINDIST, child index) argmin, k-th-MAXDIST bounds on the
+    // way, then ClosestLeaf and its right siblings until k points are seen; their
+    // points go straight into the kNN list (allowed by R4: pass 2 then treats
+    // these leaves as already scanned).
     // Pass 2 (Alg. 1 l.6-47): leftmost eligible descent, left-to-right leaf scan,
     // parent-link backtrack.
-    lvl = H;
-    node = 0;
+    bool pass1 = true;
+    int lvl = H;
+    int node = 0;
+    int pass1_lo = 0, pass1_hi = -1;
+    int64_t seen = 0;
     int visited = -1;                                            // R10
     while (true) {
         if (lvl > 0) {
             float md[V];
             S.node(internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
-            // S6: eligible(c) = MINDIST <= pd (R5) and unvisited leaves below (R8).
-            // Subtree leaf ranges are contiguous and increasing in c, so
-            // maxLeaf(child c) > visited  <=>  visited+1 < L  and
-            // base + c >= (visited+1) / F^(lvl-1)   (a warp-uniform threshold).
             const int base = node * F;
-            const int c_end = min(F, (int)ix.nlev[lvl - 1] - base);
-            const int c_min = visited + 1 < (int)ix.L ? ((visited + 1) >> ((lvl - 1) * LOGF)) - base : F;
-            unsigned mine = 0;
+            int c;
+            if (pass1) {
+                const int nb = (int)ix.nlev[lvl - 1];
+                u64 best = ~0ull;
 #pragma unroll
-            for (int t = 0; t < V; ++t) {
-                const int c = lane * V + t;
-                const bool e = c >= c_min && c < c_end && md[t] <= pd;
-                mine |= (unsigned)e << t;
+                for (int t = 0; t < V; ++t) {
+                    const int cc = lane * V + t;
+                    if (base + cc < nb) {
+                        const u64 kk = make_key(md[t], cc);
+                        best = kk < best ? kk : best;
+                    }
+                }
+                c = (int)(warp_min_u64(best) & 0xffffffffu);
+            } else {
+                // S6: eligible(c) = MINDIST <= pd (R5) and unvisited leaves below (R8).
+                // Subtree leaf ranges are contiguous and increasing in c, so
+                // maxLeaf(child c) > visited  <=>  visited+1 < L  and
+                // base + c >= (visited+1) / F^(lvl-1)   (a warp-uniform threshold).
+                const int c_end = min(F, (int)ix.nlev[lvl - 1] - base);
+                const int c_min = visited + 1 < (int)ix.L ? ((visited + 1) >> ((lvl - 1) * LOGF)) - base : F;
+                unsigned mine = 0;
+#pragma unroll
+                for (int t = 0; t < V; ++t) {
+                    const int cc = lane * V + t;
+                    const bool e = cc >= c_min && cc < c_end && md[t] <= pd;
+                    mine |= (unsigned)e << t;
+                }
+                const unsigned bal = __ballot_sync(FULL, mine != 0);
+                c = F;
+                if (bal) {                                       // leftmost (R6, R7)
+                    const int src = __ffs(bal) - 1;
+                    const unsigned m = __shfl_sync(FULL, mine, src);
+                    c = src * V + (__ffs(m) - 1);
+                }
             }
-            const unsigned bal = __ballot_sync(FULL, mine != 0);
-            if (bal) {                                           // leftmost (R6, R7)
-                const int src = __ffs(bal) - 1;
-                const unsigned m = __shfl_sync(FULL, mine, src);
-                node = base + src * V + (__ffs(m) - 1);
-                --lvl;
+            if (c < F) {
+                node = base + c;
+                if (--lvl == 0 && pass1) pass1_lo = node;        // ClosestLeaf
             } else {                                             // S7 backtrack (R9)
                 if (lvl == H) break;                             // root exhausted (R10)
                 visited = max_leaf(ix, lvl, node);
@@ -187,11 +189,22 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
         } else {
             // S8-S10: leaf j
             const int j = node;
-            bool changed;
-            if (j >= pass1_lo && j <= pass1_hi) {
-                changed = true;                                  // already offered in pass 1
-            } else {
+            bool changed = true;                                 // pass-1 leaves: already offered
+            if (pass1 || j < pass1_lo || j > pass1_hi)
                 changed = scan_leaf<D, V, KS, ST>(ix, j, q, lane, T, k, thr, S, ws.scratch);
+            if (pass1) {
+                pass1_hi = j;
+                const int64_t left = ix.n - (int64_t)j * F;
+                seen += left < F ? left : F;
+                if (seen < k && j + 1 < (int)ix.L) {
+                    node = j + 1;
+                    continue;
+                }
+                pd = fminf(pd, key_dist(thr));                   // end of pass 1: restart at the root
+                pass1 = false;
+                lvl = H;
+                node = 0;
+                continue;
             }
             pd = fminf(pd, key_dist(thr));                       // Alg. 1 l.37
             visited = j;                                         // l.38
@@ -279,6 +292,41 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
 }
 
 
+// Batch scheduling (knn_order.cu): the key of query qi is the sequence id of its
+// ClosestLeaf, reached by the greedy (MINDIST, child index) descent of PSB's pass
+// 1 (Alg. 1 l.3; R4). One warp per query, no cache, no MAXDIST.
+template <int D, int V, bool SPH>
+__global__ void __launch_bounds__(WARPS_PER_CTA * 32)
+closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, uint32_t *__restrict__ leaf_key)
+{
+    __shared__ float qs[WARPS_PER_CTA][D == 0 ? PSB_DMAX : 1];
+    constexpr int F = 32 * V;
+    const int lane = threadIdx.x & 31;
+    const int64_t qi = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
+    if (qi >= nq) return;
+    Query<D> q;
+    q.load(queries + qi * ix.d, ix.d, qs[threadIdx.x >> 5]);
+    int node = 0;
+    for (int lvl = ix.H; lvl > 0; --lvl) {
+        const float *blk = ix.nodes + ix.level_off[lvl] + (int64_t)node * ix.blk_floats;
+        float md[V], Md[V];
+        if constexpr (SPH) sphere_bounds<D, V, false>(blk, q, ix.d, lane, md, Md);
+        else node_bounds<D, V, false>(blk, q, ix.d, lane, md, Md);
+        const int base = node * F, nb = (int)ix.nlev[lvl - 1];
+        u64 best = ~0ull;
+#pragma unroll
+        for (int t = 0; t < V; ++t) {
+            const int c = lane * V + t;
+            if (base + c < nb) {
+                const u64 kk = make_key(md[t], c);
+                best = kk < best ? kk : best;
+            }
+        }
+        node = base + (int)(warp_min_u64(best) & 0xffffffffu);
+    }
+    if (lane == 0) leaf_key[qi] = (uint32_t)node;
+}
+
 // One warp per query. With `queue` non-null the grid is persistent (as many
 // CTAs as fit on the GPU) and each warp takes the next query from an atomic
 // counter when it finishes one, so a long query never holds an idle block.
@@ -287,7 +335,8 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
     __global__ void __launch_bounds__(WARPS_PER_CTA * 32, PSB_MIN_BLOCKS)                            \
     NAME(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,                          \
          int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant,             \
-         int64_t *__restrict__ stats, unsigned long long *__restrict__ queue)                        \
+         int64_t *__restrict__ stats, unsigned long long *__restrict__ queue,                        \
+         const int32_t *__restrict__ order)                                                           \
     {                                                                                                 \
         extern __shared__ __align__(16) unsigned char smem[];                                         \
         const int lane = threadIdx.x & 31;                                                            \
@@ -302,7 +351,8 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
                 qi = (int64_t)__shfl_sync(FULL, v, 0);                                                \
             }                                                                                         \
             if (qi >= nq) break;                                                                      \
-            BODY<D, V, KS, ST, SPH>(ix, queries, qi, k, out_ids, out_dists, stats, ws, use_cache, use_max, lane); \
+            const int64_t row = order ? (int64_t)__ldg(order + qi) : qi;                             \
+            BODY<D, V, KS, ST, SPH>(ix, queries, row, k, out_ids, out_dists, stats, ws, use_cache, use_max, lane); \
             if (!queue) break;                                                                        \
         }                                                                                             \
     }
@@ -471,7 +521,7 @@ static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int
     // Counting (stats) kernels are instantiated for the generic-d path only: the
     // traversal, hence every counter, does not depend on the d specialisation.
     using Kern = void (*)(DevIndex, const float *, int64_t, int, int32_t *, float *, uint32_t, int64_t *,
-                          unsigned long long *);
+                          unsigned long long *, const int32_t *);
     Kern kern;
     const bool psbk = algo == PSB_ALGO_PSB;
     if constexpr (D == 0) {
@@ -519,23 +569,53 @@ static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int
         cudaFreeAsync(gpd, st);
         return rc;
     }
+    // Batch scheduling: process the queries in the order of their closest leaf
+    // (knn_order.cu) so concurrent warps share leaves in L1/L2. Rows are written
+    // to their input positions, so results are unchanged.
+    int32_t *order = nullptr;
+    const double leaf_bytes = (double)ix.L * ix.F * (ix.d * 4 + 4);
+    const bool reorder = (variant & PSB_VAR_LEAF_ORDER) ||
+                         (!(variant & PSB_VAR_INPUT_ORDER) && nq >= REORDER_MIN_QUERIES && leaf_bytes >= REORDER_MIN_BYTES);
+    if (reorder) {
+        uint32_t *leaf_key = nullptr;
+        if ((e = cudaMallocFromPoolAsync((void **)&leaf_key, (size_t)nq * 4, pool, st)) != cudaSuccess ||
+            (e = cudaMallocFromPoolAsync((void **)&order, (size_t)nq * 4, pool, st)) != cudaSuccess) {
+            if (leaf_key) cudaFreeAsync(leaf_key, st);
+            return report_cuda(e, "cudaMallocFromPoolAsync (query order)");
+        }
+        auto ck = ix.sphere ? closest_leaf_kernel<D, V, true> : closest_leaf_kernel<D, V, false>;
+        ck<<<(unsigned)((nq + WARPS_PER_CTA - 1) / WARPS_PER_CTA), WARPS_PER_CTA * 32, 0, st>>>(ix, queries, nq,
+                                                                                               leaf_key);
+        int rc = report_cuda(cudaGetLastError(), "closest-leaf kernel launch");
+        if (rc == PSB_OK) rc = sort_query_order(leaf_key, nq, ix.L, order, pool, st);
+        cudaFreeAsync(leaf_key, st);
+        if (rc != PSB_OK) {
+            cudaFreeAsync(order, st);
+            return rc;
+        }
+    }
     // More queries than resident warps: persistent grid + atomic query queue.
     int per_sm = 0;
     unsigned long long *queue = nullptr;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, WARPS_PER_CTA * 32, smem) == cudaSuccess &&
         per_sm > 0 && blocks > (int64_t)per_sm * ix.sm_count) {
-        if ((e = cudaMallocFromPoolAsync((void **)&queue, sizeof(unsigned long long), pool, st)) != cudaSuccess)
+        if ((e = cudaMallocFromPoolAsync((void **)&queue, sizeof(unsigned long long), pool, st)) != cudaSuccess) {
+            if (order) cudaFreeAsync(order, st);
             return report_cuda(e, "cudaMallocFromPoolAsync (query queue)");
+        }
         if ((e = cudaMemsetAsync(queue, 0, sizeof(unsigned long long), st)) != cudaSuccess) {
             cudaFreeAsync(queue, st);
+            if (order) cudaFreeAsync(order, st);
             return report_cuda(e, "cudaMemsetAsync (query queue)");
         }
         blocks = (int64_t)per_sm * ix.sm_count;
     }
     cudaGetLastError();
-    kern<<<(unsigned)blocks, WARPS_PER_CTA * 32, smem, st>>>(ix, queries, nq, k, oi, od, variant, stats, queue);
+    kern<<<(unsigned)blocks, WARPS_PER_CTA * 32, smem, st>>>(ix, queries, nq, k, oi, od, variant, stats, queue,
+                                                             order);
     int rc = report_cuda(cudaGetLastError(), "tree kernel launch");
     if (queue) cudaFreeAsync(queue, st);
+    if (order) cudaFreeAsync(order, st);
     return rc;
 }
 

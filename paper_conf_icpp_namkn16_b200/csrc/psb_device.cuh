@@ -258,6 +258,7 @@ __device__ __forceinline__ float kth_bound(const float (&Md)[V], int k, float pd
     c = __reduce_add_sync(FULL, c);
     if (c < k) return pd;
     uint32_t res = 0;
+#pragma unroll 1
     for (int bit = 30; bit >= 0; --bit) {
         const uint32_t trial = res | (1u << bit);
         int n = 0;
@@ -365,6 +366,9 @@ struct TopK {
     template <int V>
     __device__ __forceinline__ int offer(const u64 (&cand)[V], int k, int lane, u64 &thr, u64 *scratch)
     {
+        // Code size matters here (the kernels are instruction-cache bound at
+        // small d, profiles/r01_icache.md): every insertion / merge network below
+        // has exactly one inlined copy per call site of offer().
         unsigned bal[V];
         int m = 0;
 #pragma unroll
@@ -374,44 +378,47 @@ struct TopK {
         }
         if (m == 0) return 0;
         if (m <= 2) {
+            for (int i = 0; i < m; ++i) {                // (t, lane) order; warp-uniform
+                int t0 = 0;                                  // first t with a pending candidate
+                unsigned b = bal[0];
 #pragma unroll
-            for (int t = 0; t < V; ++t) {
-                unsigned b = bal[t];
-                while (b) {
-                    const int src = __ffs(b) - 1;
-                    b &= b - 1;
-                    const u64 x = __shfl_sync(FULL, cand[t], src);
-                    if (x < thr) {
-                        insert(x, lane);
-                        thr = kth(k);
-                    }
+                for (int t = V - 1; t >= 0; --t)
+                    if (bal[t]) { t0 = t; b = bal[t]; }
+                const int src = __ffs(b) - 1;
+                u64 v = cand[0];
+#pragma unroll
+                for (int t = 1; t < V; ++t)
+                    if (t == t0) v = cand[t];
+#pragma unroll
+                for (int t = 0; t < V; ++t)
+                    if (t == t0) bal[t] &= bal[t] - 1;
+                const u64 x = __shfl_sync(FULL, v, src);
+                if (x < thr) {
+                    insert(x, lane);
+                    thr = kth(k);
                 }
             }
             return m;
         }
-        if (m <= 32) {
-            const unsigned lt = (1u << lane) - 1;
-            int base = 0;
+        // Compact the candidates in (t, lane) order through 32 u64 of scratch and
+        // merge them 32 at a time (m <= 32*V). A candidate that is no longer below
+        // the k-th key after an earlier round only lands at positions >= k.
+        const unsigned lt = (1u << lane) - 1;
+        for (int r = 0; r < m; r += 32) {
+            int base = -r;
 #pragma unroll
             for (int t = 0; t < V; ++t) {
-                if (bal[t] >> lane & 1u) scratch[base + __popc(bal[t] & lt)] = cand[t];
+                const int i = base + __popc(bal[t] & lt);
+                if ((bal[t] >> lane & 1u) && i >= 0 && i < 32) scratch[i] = cand[t];
                 base += __popc(bal[t]);
             }
             __syncwarp();
-            const u64 c = lane < m ? scratch[lane] : ~0ull;
+            const int n = min(m - r, 32);
+            const u64 c = lane < n ? scratch[lane] : ~0ull;
             __syncwarp();
-            if (m <= 8) merge32<8>(c, lane);
-            else if (m <= 16) merge32<16>(c, lane);
+            if (n <= 8) merge32<8>(c, lane);
+            else if (n <= 16) merge32<16>(c, lane);
             else merge32<32>(c, lane);
-        } else {
-#pragma unroll
-            for (int t = 0; t < V; ++t) {
-                const u64 c = cand[t] < thr ? cand[t] : ~0ull;
-                if (__any_sync(FULL, c != ~0ull)) {
-                    merge32(c, lane);
-                    thr = kth(k);
-                }
-            }
         }
         thr = kth(k);
         return m;

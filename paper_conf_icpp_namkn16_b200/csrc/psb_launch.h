@@ -47,6 +47,11 @@ int launch_brute_v(const DevIndex &ix, const float *queries, int64_t nq, int k, 
 int gpu_bulk_load(const float *d_points, const GpuLayoutShape &sh, int64_t id_base, float *pts, int32_t *ids,
                   float *nodes, cudaStream_t st, bool sphere, int kmeans_iters);
 
+// Stable sort of queries by closest-leaf id (knn_order.cu): order[i] = the input
+// row processed i-th. leaf_key is [nq] device memory; order is [nq].
+int sort_query_order(const uint32_t *leaf_key, int64_t nq, int64_t L, int32_t *order, cudaMemPool_t pool,
+                     cudaStream_t st);
+
 // [parts][nq][k] sorted (dist, id) lists -> first k of their union (knn_brute.cu).
 int launch_merge(const int32_t *ids, const float *dists, int parts, int64_t nq, int k, int32_t *oi,
                  float *od, cudaStream_t st);

@@ -109,6 +109,37 @@ def test_c2_nocache_and_batches(c2):
     assert_same(r, (exp[0][::-1][:2000], exp[1][::-1][:2000]), "C2 reversed")
 
 
+@pytest.mark.parametrize("algo", ["psb", "bnb"])
+def test_c2_query_order_independent(c2, algo):
+    """Batch scheduling (closest-leaf order, default for >= 1024 queries) and input
+    order return the same rows, both equal to the oracle; also a ragged batch just
+    above the reorder threshold and one with duplicated queries."""
+    psb = _psb()
+    cfg, pts, qs, idx, exp = c2
+    sl = slice(0, 5000)
+    assert_same(run(idx, qs[sl], cfg.k, algo, psb.PSB_VAR_INPUT_ORDER), (exp[0][sl], exp[1][sl]), "input order")
+    lo = psb.PSB_VAR_LEAF_ORDER
+    assert_same(run(idx, qs[sl], cfg.k, algo, lo), (exp[0][sl], exp[1][sl]), "leaf order")
+    assert_same(run(idx, qs[sl], cfg.k, algo, lo | 1), (exp[0][sl], exp[1][sl]), "leaf order, no cache")
+    sel = np.r_[np.arange(1025), np.arange(7)]          # 1032 queries, 7 repeated
+    assert_same(run(idx, qs[sel], cfg.k, algo, lo), (exp[0][sel], exp[1][sel]), "ragged + duplicates")
+    assert_same(run(idx, qs[:3], cfg.k, algo, lo), (exp[0][:3], exp[1][:3]), "tiny batch")
+
+
+def test_query_order_generic_d_and_sphere():
+    """The reorder pre-pass on the runtime-d kernels (d=5) and on sphere nodes."""
+    psb = _psb()
+    rng = np.random.default_rng(7)
+    pts = rng.random((60000, 5), dtype=np.float32)
+    qs = rng.random((1500, 5), dtype=np.float32)
+    exp = oracle.knn_bruteforce(pts, qs, 10)
+    for flags in (0, psb.PSB_NODE_SPHERE):
+        idx = psb.psb_build_ex(pts, 64, packing=flags)
+        for algo in ("psb", "bnb"):
+            assert_same(run(idx, qs, 10, algo, psb.PSB_VAR_LEAF_ORDER), exp, f"d=5 flags={flags} {algo}")
+        idx.free()
+
+
 def test_c3_sampled():
     """configs[2]: 8-D uniform n=4M F=128 k=16; a 2,000-query sample of the 10^5."""
     cfg = W.config("C3")
@@ -303,6 +334,9 @@ def test_host_buffers_and_stats(c2):
         i2, _, st2 = psb.psb_knn_stats(idx, qd, cfg.k, algo=algo)
         torch.cuda.synchronize()
         assert np.array_equal(st2.cpu().numpy(), got[0])          # deterministic
+        _, _, st3 = psb.psb_knn_stats(idx, qd, cfg.k, algo=algo, variant=psb.PSB_VAR_LEAF_ORDER)
+        torch.cuda.synchronize()
+        assert np.array_equal(st3.cpu().numpy(), got[0])          # same traversal in any query order
         assert (got[1][:, 3] == 0).all()                           # no cache -> no hits
         assert np.array_equal(got[0][:, 0] + got[0][:, 3], got[1][:, 0])  # same visits, cache or not
         assert np.array_equal(got[0][:, 1], got[1][:, 1])          # same leaves scanned
