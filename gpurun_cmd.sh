@@ -1,5 +1,6 @@
-mkdir -p gpurun_out/ncu
 for c in C2 C3 C5; do
-timeout 900 ncu --set full --import-source on --clock-control none -k regex:psb_kernel --launch-skip 1 -c 1 -f -o gpurun_out/ncu/${c}_psb_v2 python tools/prof_one.py $c psb > gpurun_out/ncu/${c}_psb_v2.log 2>&1
-tail -1 gpurun_out/ncu/${c}_psb_v2.log
-done
+for a in psb bnb; do
+PSB_LIB_PATH=$PWD/ab/libpsb_prev.so timeout 300 python tools/var_ab.py $c $a 0 2>&1 | grep -v Warn | sed 's/^/PREV /'
+timeout 300 python tools/var_ab.py $c $a 0 2>&1 | grep -v Warn
+done; done
+timeout 1200 python -m pytest tests -m gpu -q -x 2>&1 | tail -2

@@ -275,7 +275,8 @@ __device__ __forceinline__ float kth_bound(const float (&Md)[V], int k, float pd
 __device__ __forceinline__ u64 cmpx(u64 v, int j, bool take_min)
 {
     const u64 o = __shfl_xor_sync(FULL, v, j);
-    return take_min ? (o < v ? o : v) : (o < v ? v : o);
+    // one u64 compare and one select (o == v only for equal fillers: either is right)
+    return (o < v) == take_min ? o : v;
 }
 // Sorts each group of G lanes (G = 8, 16 or 32; groups alternate direction).
 // With candidates in lanes 0..G-1 and ~0 everywhere else, the whole warp is
