@@ -49,6 +49,8 @@ def parse():
     ap.add_argument("--mode", default="query", choices=["query", "data"])
     ap.add_argument("--slab", type=int, default=0,
                     help="data mode on ONE GPU: run rank 0's local step of a P-way data-sharded job")
+    ap.add_argument("--exchange", default="p2p", choices=["p2p", "nccl"],
+                    help="data mode, N>1: merge straight from peer memory (psb_exchange) or NCCL all-gather + merge")
     ap.add_argument("--algo", default="psb", choices=["psb", "bnb", "brute"])
     ap.add_argument("--variant", type=int, default=0)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -190,6 +192,22 @@ def run_reference(args, rank, world):
 
 
 # ----------------------------------------------------------------------------- our arm
+def count_launches(step):
+    """Kernels one step launches, counted by the CUDA profiler (CUPTI via
+    torch.profiler) on an untimed extra step: {name: count} and the total."""
+    import torch
+    from torch.profiler import ProfilerActivity, profile
+    with profile(activities=[ProfilerActivity.CUDA]) as prof:
+        step()
+        torch.cuda.synchronize()
+    names = {}
+    for ev in prof.events():
+        if ev.device_type == torch.autograd.DeviceType.CUDA and not ev.name.startswith(("Memcpy", "Memset")):
+            short = ev.name.split("(")[0].replace("void ", "")
+            names[short] = names.get(short, 0) + 1
+    return sum(names.values()), names
+
+
 def main():
     args = parse()
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -203,9 +221,15 @@ def main():
     import paper_conf_icpp_namkn16_b200 as psb
     from paper_conf_icpp_namkn16_b200 import dist as pdist
 
-    torch.cuda.set_device(local)
+    # PSB_BENCH_DEVICE / PSB_DIST_BACKEND: test hooks (several ranks on one GPU over gloo)
+    torch.cuda.set_device(int(os.environ.get("PSB_BENCH_DEVICE", local)))
+    backend = os.environ.get("PSB_DIST_BACKEND", "nccl")
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", torch.cuda.current_device()))
+        else:
+            dist.init_process_group(backend)
+    red_dev = "cuda" if backend == "nccl" else "cpu"
     if args.profile:
         args.no_extras = True
         args.no_cpu_baseline = True
@@ -246,15 +270,22 @@ def main():
         return psb.psb_knn_ex(idx, qq, kk, algo=algo, variant=args.variant,
                               out=(out_i, out_d) if qq.shape[0] == q else None)
 
+    ex = None
+    if args.mode == "data" and world > 1 and args.exchange == "p2p":
+        ex = pdist.peer_exchange(q, k)
+
     def step():
         if args.mode == "query" or world == 1:
             local_knn(qd, k)
+        elif ex is not None:
+            pdist.data_sharded_knn_p2p(ex, idx, qd, algo=algo, variant=args.variant)
         else:
             pdist.data_sharded_knn(local_knn, pdist.device_merge, qd, k)
 
     for _ in range(max(3, args.warmup)):
         step()
     torch.cuda.synchronize()
+    launches_per_step, launch_names = count_launches(step)
 
     sampler = ClockSampler(local)
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
@@ -274,7 +305,7 @@ def main():
     if world > 1:
         dist.barrier()
     step_ms = [a.elapsed_time(b) for a, b in evs]
-    total_ms = torch.tensor([sum(step_ms)], dtype=torch.float64, device="cuda")
+    total_ms = torch.tensor([sum(step_ms)], dtype=torch.float64, device=red_dev)
     if world > 1:
         dist.all_reduce(total_ms, op=dist.ReduceOp.MAX)
     total_ms = float(total_ms.item())
@@ -301,7 +332,7 @@ def main():
             stream.synchronize()
             if i >= max(3, args.warmup):
                 e2e_ms.append((time.perf_counter() - t0) * 1e3)
-        e2e_t = torch.tensor([sum(e2e_ms)], dtype=torch.float64, device="cuda")
+        e2e_t = torch.tensor([sum(e2e_ms)], dtype=torch.float64, device=red_dev)
         if world > 1:
             dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
         extras["e2e"] = {"value": units * args.steps / (float(e2e_t.item()) / 1e3), "unit": UNIT,
@@ -375,7 +406,9 @@ def main():
             "data": "synthetic (workloads/: seeded SplitMix64 uniform / 100-cluster Gaussian)",
             "config": {**cfg.describe(), "q": q, "algo": args.algo, "variant": args.variant,
                        "parallelism": (f"query-sharded x{world} (replicated index)" if args.mode == "query"
-                                       else (f"data-sharded x{world} (NCCL all-gather + merge)" if world > 1 else
+                                       else ((f"data-sharded x{world} (merge from peer memory, psb_exchange)"
+                                              if ex is not None else f"data-sharded x{world} (NCCL all-gather + merge)")
+                                             if world > 1 else
                                              f"data-sharded slab 0 of {max(1, args.slab)} (local step only, 1 GPU)")),
                        "points_on_this_gpu": int(pts.shape[0]),
                        "l2": "flushed between steps (256 MiB write)", "index_bytes": idx.device_bytes},
@@ -389,12 +422,18 @@ def main():
                                                  "changing_leaf_scans": stats_sum[4] / q,
                                                  "keys_merged": stats_sum[5] / q})},
             "clocks": clocks,
-            "gpu_launches": args.steps * (1 if args.algo != "brute" else 2) * (1 if args.mode == "query" or world == 1 else 2),
+            "gpu_launches": args.steps * launches_per_step,
+            "gpu_launch_names": launch_names,
             **extras,
         }
         if cpu is not None:
             line["cpu_baseline"] = cpu
         print(json.dumps(line), flush=True)
+    if ex is not None:
+        if ex.timed_out():
+            raise RuntimeError("psb_exchange: a peer wait timed out")
+        dist.barrier()
+        ex.free()
     idx.free()
     if world > 1:
         dist.destroy_process_group()

@@ -1,6 +1,4 @@
-for c in C2 C3 C5; do
-for a in psb bnb; do
-PSB_LIB_PATH=$PWD/ab/libpsb_prev.so timeout 300 python tools/var_ab.py $c $a 0 2>&1 | grep -v Warn | sed 's/^/PREV /'
-timeout 300 python tools/var_ab.py $c $a 0 2>&1 | grep -v Warn
-done; done
-timeout 1200 python -m pytest tests -m gpu -q -x 2>&1 | tail -2
+O=gpurun_out/r01d; mkdir -p $O
+timeout 900 python -m pytest tests/test_gpu_exchange.py -q -x 2>&1 | tail -15
+PSB_DIST_BACKEND=gloo PSB_BENCH_DEVICE=0 timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --mode data --config C2 --steps 20 --warmup 3 --no-extras > $O/bench_data2_p2p_1gpu.json 2> $O/bench_data2_p2p_1gpu.err
+tail -3 $O/bench_data2_p2p_1gpu.err; cat $O/bench_data2_p2p_1gpu.json | head -c 1500

@@ -181,6 +181,42 @@ int psb_knn_stats(const psb_index *idx, const float *queries, int64_t q, int32_t
 int psb_merge_topk(const int32_t *ids, const float *dists, int32_t parts, int64_t q, int32_t k,
                    int32_t *out_ids, float *out_dists, void *stream);
 
+/* ---- Data-sharded exchange over peer memory (north_star) ----
+ * The NCCL route (all-gather of every shard's [q][k] lists + psb_merge_topk) is
+ * replaced by one kernel per step that pulls only the rows a rank owns directly
+ * out of the peers' result buffers (CUDA IPC mappings over NVLink/NVSwitch) and
+ * merges them, after a device-side flag barrier: no collective launch, no
+ * staging buffer, P-fold less traffic into each rank than an all-gather.
+ *
+ * Protocol, one object per rank (all ranks: same parts, q, k):
+ *   psb_exchange_create(parts, rank, q, k, &x)   allocates on the current device
+ *     two [q][k] result buffers (alternating by epoch parity) and parts flag slots;
+ *   psb_exchange_handle(x, blob, cap, &used)     blob (IPC handles) to share with
+ *     every rank (e.g. torch.distributed all_gather_object);
+ *   psb_exchange_connect(x, blobs)               maps all ranks' buffers (blobs in
+ *     rank order; a blob from the calling process is used without IPC);
+ *   each step, with epoch = 1, 2, 3 ...:
+ *     psb_exchange_buffers(x, epoch, &ids, &dists)  this rank's result buffers for
+ *       the step: run the local psb_knn* into them (ids global via id_base);
+ *     psb_exchange_step(x, epoch, row0, rows, out_ids, out_dists, stream)
+ *       stream-ordered after the local search: signals every peer, waits (on the
+ *       device) until every peer has signalled `epoch`, then writes the merged
+ *       first k of rows [row0, row0+rows) of all parts' lists to out[rows][k].
+ *   psb_exchange_status(x, &timed_out)           1 if a wait gave up after 10 s
+ *     (a peer never signalled; that step's output is undefined).
+ * Every rank must call psb_exchange_step for every epoch. k <= 128,
+ * parts <= PSB_MAX_PARTS. Synchronous except psb_exchange_step. */
+#define PSB_MAX_PARTS 16
+typedef struct psb_exchange psb_exchange; /* opaque */
+int psb_exchange_create(int32_t parts, int32_t rank, int64_t q, int32_t k, psb_exchange **out);
+int psb_exchange_handle(const psb_exchange *x, void *blob, int64_t cap, int64_t *used);
+int psb_exchange_connect(psb_exchange *x, const void *const *blobs);
+int psb_exchange_buffers(const psb_exchange *x, int64_t epoch, int32_t **ids, float **dists);
+int psb_exchange_step(psb_exchange *x, int64_t epoch, int64_t row0, int64_t rows, int32_t *out_ids,
+                      float *out_dists, void *stream);
+int psb_exchange_status(const psb_exchange *x, int32_t *timed_out);
+void psb_exchange_free(psb_exchange *x);
+
 /* Shape of an index. Any output pointer may be NULL. `levels` counts internal
  * levels (root at level `levels`, leaves at level 0); device_bytes is the index's
  * device footprint. */

@@ -27,13 +27,15 @@ PSB_BUILD_HOST = 0x100
 PSB_NODE_SPHERE = 0x200
 PSB_ALGO_PSB, PSB_ALGO_BNB, PSB_ALGO_BRUTE = 0, 1, 2
 PSB_VAR_NOCACHE, PSB_VAR_NOMAXDIST, PSB_VAR_INPUT_ORDER, PSB_VAR_LEAF_ORDER = 1, 2, 4, 8
-PSB_KMAX, PSB_DMAX = 2048, 64
+PSB_KMAX, PSB_DMAX, PSB_MAX_PARTS = 2048, 64, 16
 FANOUTS = (32, 64, 128, 256, 512)
 
 # every symbol include/psb.h declares (tests check the .so exports all of them)
 EXPORTS = ("psb_build", "psb_build_ex", "psb_knn", "psb_knn_branch_and_bound", "psb_knn_bruteforce",
            "psb_knn_ex", "psb_knn_stats", "psb_knn_split", "psb_merge_topk", "psb_index_info", "psb_index_export", "psb_build_host_blob",
-           "psb_free", "psb_last_error", "psb_version")
+           "psb_free", "psb_last_error", "psb_version", "psb_exchange_create", "psb_exchange_handle",
+           "psb_exchange_connect", "psb_exchange_buffers", "psb_exchange_step", "psb_exchange_status",
+           "psb_exchange_free")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libpsb.so not built at {LIB_PATH}: run __graft_entry__.build() "
@@ -56,6 +58,13 @@ _sig = {
     "psb_index_export": (ctypes.c_int, [_vp, _vp, _i64, _P(_i64)]),
     "psb_build_host_blob": (ctypes.c_int, [_vp, _i64, _i32, _i32, _i64, _u32, _vp, _i64, _P(_i64)]),
     "psb_free": (None, [_vp]),
+    "psb_exchange_create": (ctypes.c_int, [_i32, _i32, _i64, _i32, _P(_vp)]),
+    "psb_exchange_handle": (ctypes.c_int, [_vp, _vp, _i64, _P(_i64)]),
+    "psb_exchange_connect": (ctypes.c_int, [_vp, _P(_vp)]),
+    "psb_exchange_buffers": (ctypes.c_int, [_vp, _i64, _P(_vp), _P(_vp)]),
+    "psb_exchange_step": (ctypes.c_int, [_vp, _i64, _i64, _i64, _vp, _vp, _vp]),
+    "psb_exchange_status": (ctypes.c_int, [_vp, _P(_i32)]),
+    "psb_exchange_free": (None, [_vp]),
     "psb_last_error": (ctypes.c_char_p, []),
     "psb_version": (ctypes.c_char_p, []),
 }
@@ -246,6 +255,72 @@ def psb_merge_topk(ids, dists, k: int, stream=None, out=None):
     _check(_lib.psb_merge_topk(ids.data_ptr(), dists.data_ptr(), parts, q, k, out[0].data_ptr(),
                                out[1].data_ptr(), _stream_handle(stream)), "psb_merge_topk")
     return out
+
+
+class Exchange:
+    """Data-sharded exchange over peer memory (include/psb.h psb_exchange_*): this
+    rank's double-buffered [q, k] result lists and flag slots, mapped by every
+    rank; `step` merges the rows this rank owns straight out of all ranks' lists."""
+
+    def __init__(self, parts: int, rank: int, q: int, k: int):
+        h = ctypes.c_void_p()
+        _check(_lib.psb_exchange_create(parts, rank, q, k, ctypes.byref(h)), "psb_exchange_create")
+        self._h, self.parts, self.rank, self.q, self.k = h, parts, rank, q, k
+        self.epoch = 0
+
+    def handle(self) -> bytes:
+        used = _i64()
+        _check(_lib.psb_exchange_handle(self._h, None, 0, ctypes.byref(used)), "psb_exchange_handle")
+        buf = ctypes.create_string_buffer(used.value)
+        _check(_lib.psb_exchange_handle(self._h, buf, used.value, ctypes.byref(used)), "psb_exchange_handle")
+        return buf.raw
+
+    def connect(self, blobs):
+        """blobs: every rank's handle() in rank order."""
+        keep = [ctypes.create_string_buffer(b, len(b)) for b in blobs]
+        arr = (_vp * len(keep))(*[ctypes.cast(b, _vp) for b in keep])
+        _check(_lib.psb_exchange_connect(self._h, arr), "psb_exchange_connect")
+
+    def begin(self):
+        """Next epoch; returns (ids_ptr, dists_ptr) of this rank's [q, k] result buffers for it."""
+        self.epoch += 1
+        pi, pd = _vp(), _vp()
+        _check(_lib.psb_exchange_buffers(self._h, self.epoch, ctypes.byref(pi), ctypes.byref(pd)),
+               "psb_exchange_buffers")
+        return pi.value, pd.value
+
+    def local_knn(self, index: "Index", queries, algo: int = PSB_ALGO_PSB, variant: int = 0, stream=None):
+        """begin() + this rank's local search (all q queries, device buffers) into its buffers."""
+        assert queries.is_cuda and queries.shape[0] == self.q
+        pi, pd = self.begin()
+        _check(_lib.psb_knn_ex(index.handle, queries.data_ptr(), self.q, self.k, pi, pd, _stream_handle(stream),
+                               algo, variant), "psb_knn_ex (exchange)")
+
+    def step(self, row0: int, rows: int, stream=None, out=None):
+        """Signal the peers, wait for all of them (on the device), merge rows [row0, row0+rows)."""
+        torch = _torch()
+        if out is None:
+            out = (torch.empty((rows, self.k), dtype=torch.int32, device="cuda"),
+                   torch.empty((rows, self.k), dtype=torch.float32, device="cuda"))
+        _check(_lib.psb_exchange_step(self._h, self.epoch, row0, rows, out[0].data_ptr(), out[1].data_ptr(),
+                                      _stream_handle(stream)), "psb_exchange_step")
+        return out
+
+    def timed_out(self) -> bool:
+        v = _i32()
+        _check(_lib.psb_exchange_status(self._h, ctypes.byref(v)), "psb_exchange_status")
+        return bool(v.value)
+
+    def free(self):
+        if self._h is not None and self._h.value:
+            _lib.psb_exchange_free(self._h)
+        self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
 
 
 def _parse_blob(buf: np.ndarray) -> dict:

@@ -18,9 +18,13 @@ constexpr int WARPS_PER_CTA = 4;
 // anyway (profiles/r01_query_order.md: a loss at C2's 16 MB, a gain from C3's 146 MB).
 constexpr int64_t REORDER_MIN_QUERIES = 1024;
 constexpr double REORDER_MIN_BYTES = 64.0 * (1 << 20);
-#ifndef PSB_MIN_BLOCKS
-#define PSB_MIN_BLOCKS 8   // <= 64 registers: measured best on C2/C3 (profiles/r01_occupancy.md)
-#endif
+// Resident CTAs per SM the traversal kernels are compiled for (register cap
+// 65536 / (128 * blocks)): 8 (<= 64 registers) measured best at d <= 8, 6 (<= 80)
+// at d = 16 and for the runtime-d kernels (profiles/r01_occupancy.md).
+template <int D>
+struct MinBlocks {
+    static constexpr int value = (D == 0 || D >= 16) ? 6 : 8;
+};
 
 struct WarpState {
     float *cache_md;     // [(H+1)][F] child MINDISTs of the node cached per level
@@ -332,7 +336,7 @@ closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, 
 // counter when it finishes one, so a long query never holds an idle block.
 #define PSB_TREE_KERNEL(NAME, BODY)                                                                  \
     template <int D, int V, int KS, bool ST, bool SPH>                                                \
-    __global__ void __launch_bounds__(WARPS_PER_CTA * 32, PSB_MIN_BLOCKS)                            \
+    __global__ void __launch_bounds__(WARPS_PER_CTA * 32, MinBlocks<D>::value)                       \
     NAME(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,                          \
          int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant,             \
          int64_t *__restrict__ stats, unsigned long long *__restrict__ queue,                        \
@@ -497,7 +501,7 @@ __device__ __forceinline__ void psb_part_query(const DevIndex &ix, const float *
 }
 
 template <int D, int V, int KS, bool ST, bool SPH>
-__global__ void __launch_bounds__(WARPS_PER_CTA * 32, PSB_MIN_BLOCKS)
+__global__ void __launch_bounds__(WARPS_PER_CTA * 32, MinBlocks<D>::value)
 psb_split_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int parts, int k,
                  int32_t *__restrict__ part_ids, float *__restrict__ part_dists, float *__restrict__ gpd,
                  uint32_t variant)

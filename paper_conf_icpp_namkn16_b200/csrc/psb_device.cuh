@@ -19,6 +19,9 @@
 namespace psb {
 
 typedef unsigned long long u64;
+#ifndef PSB_INSERT_MAX
+#define PSB_INSERT_MAX 2   // up to this many candidates are inserted one by one, more are merged
+#endif
 constexpr unsigned FULL = 0xffffffffu;
 // (dist, id) packed as one u64 key: for dist >= +0 the IEEE bit pattern orders
 // like the value, so u64 order == lexicographic (dist, id) order for ids >= 0.
@@ -378,7 +381,7 @@ struct TopK {
             m += __popc(bal[t]);
         }
         if (m == 0) return 0;
-        if (m <= 2) {
+        if (m <= PSB_INSERT_MAX) {
             for (int i = 0; i < m; ++i) {                // (t, lane) order; warp-uniform
                 int t0 = 0;                                  // first t with a pending candidate
                 unsigned b = bal[0];

@@ -8,7 +8,9 @@ combined with an NCCL all-gather over NVLink plus an on-device k-way merge."
 
 Everything here is plumbing: the local search and the merge are the library's
 CUDA kernels (``psb_knn`` / ``psb_merge_topk``); the collective is NCCL via
-``torch.distributed``. The orchestration functions take the local-search and
+``torch.distributed``. ``data_sharded_knn_p2p`` is the collective-free route:
+the library's exchange kernel pulls each rank's rows from its peers' result
+buffers over NVLink (CUDA IPC), torch.distributed only swaps the handles once. The orchestration functions take the local-search and
 merge steps as callables so their host logic can be tested on CPU with gloo.
 """
 from __future__ import annotations
@@ -84,6 +86,30 @@ def query_sharded_knn(local_knn: Callable, queries: torch.Tensor, k: int, group=
     gi, gd = allgather_topk(pad_i, pad_d, group)
     return (torch.cat([gi[r, : sizes[r]] for r in range(world)]),
             torch.cat([gd[r, : sizes[r]] for r in range(world)]))
+
+
+def peer_exchange(q: int, k: int, group=None):
+    """Set up this rank's psb_exchange (include/psb.h): create it, share its IPC
+    handle blob with every rank (all_gather_object: host bytes, once), map the
+    peers' buffers. Collective over `group`."""
+    from . import Exchange
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    ex = Exchange(world, rank, q, k)
+    blobs = [None] * world
+    dist.all_gather_object(blobs, ex.handle(), group=group)
+    ex.connect(blobs)
+    return ex
+
+
+def data_sharded_knn_p2p(ex, index, queries: torch.Tensor, algo: int = 0, variant: int = 0, stream=None):
+    """One data-sharded step without a collective: local search into this rank's
+    exchange buffers, then one kernel that waits for every peer's flag and merges
+    this rank's query slice straight out of all ranks' buffers over NVLink.
+    Returns (ids, dists) for the slice query_slice(q, world, rank)."""
+    ex.local_knn(index, queries, algo=algo, variant=variant, stream=stream)
+    sl = query_slice(ex.q, ex.parts, ex.rank)
+    return ex.step(sl.start, sl.stop - sl.start, stream=stream)
 
 
 def build_shard(points, fanout: int, world: int, rank: int, packing: int = 0):
