@@ -555,6 +555,11 @@ __device__ __forceinline__ bool scan_leaf(const DevIndex &ix, int leaf, const Qu
     constexpr int F = 32 * V;
     float dist[V];
     S.scan();
+#if PSB_PREFETCH_NEXT
+    // speculative: the right sibling is next whenever this scan changes the list
+    if (leaf + 1 < ix.L && lane < ix.d * V)
+        asm volatile("prefetch.global.L1 [%0];" ::"l"(ix.pts + ((int64_t)leaf + 1) * ix.d * F + lane * 32));
+#endif
     leaf_dists<D, V>(ix.pts + (int64_t)leaf * ix.d * F, q, ix.d, lane, dist);
     const float td = key_dist(thr);
     bool any = false;

@@ -124,6 +124,9 @@ def main():
             md.append("")
         d0 = ls[0]
         traffic[tag] = {"dram_bytes_per_launch": d0.get("dram_read", 0) + d0.get("dram_write", 0),
+                        "l2_bytes_per_launch": d0.get("l2_bytes"),
+                        "warp_inst_per_launch": d0.get("warp_inst"),
+                        "issue_active_pct": d0.get("issue_active_pct"),
                         "source": f"profiles/{a.round}_ncu.md ({os.path.basename(rep)})",
                         "note": "ncu flushes caches before the replayed launch (cold)"}
     open(os.path.join(ROOT, "profiles", f"{a.round}_ncu.md"), "w").write("\n".join(md) + "\n")
