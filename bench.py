@@ -295,10 +295,21 @@ def main():
     if algo == psb.PSB_ALGO_BRUTE:
         alg_bytes = idx.leaves * idx.fanout * (idx.d * 4) * q + q * (4 * idx.d + 8 * k)
         stats_sum = None
+        in_batch = None
     else:
         _, _, st = psb.psb_knn_stats(idx, qd, k, algo=algo, variant=args.variant, out=(out_i, out_d))
-        stats_sum = st.sum(0).tolist()
+        stn = st.cpu().numpy()
+        stats_sum = stn[:, :6].sum(0).tolist()
         alg_bytes = psb.algorithmic_bytes(idx, stats_sum, q, k)
+        # in-batch service time per query (%globaltimer stamps of the counting launch,
+        # SURVEY §8(d) latency (b)); the counting kernel is the runtime-d instantiation
+        svc = np.sort((stn[:, 7] - stn[:, 6]) / 1e3)
+        span = (stn[:, 7].max() - stn[:, 6].min()) / 1e3
+        last_start = (stn[:, 6].max() - stn[:, 6].min()) / 1e3
+        in_batch = {"p50": float(svc[len(svc) // 2]), "p99": float(svc[min(len(svc) - 1, int(len(svc) * 0.99))]),
+                    "max": float(svc[-1]), "batch_span_us": float(span), "last_query_start_us": float(last_start),
+                    "definition": "per-query service time inside one batch launch (%globaltimer when the warp "
+                                  "took / finished the query), counting-kernel instantiation"}
 
     def local_knn(qq, kk):
         return psb.psb_knn_ex(idx, qq, kk, algo=algo, variant=args.variant,
@@ -401,7 +412,7 @@ def main():
             "brute": lat_of(lambda x: psb.psb_knn_ex(idx, x, k, algo=psb.PSB_ALGO_BRUTE, out=(h1i, h1d)),
                             min(nl, 50)),
         }
-        extras["latency_us"] = {**lats[args.algo], "by_algo": lats,
+        extras["latency_us"] = {**lats[args.algo], "by_algo": lats, "in_batch": in_batch,
                                 "definition": "one query per call, launch to results in pinned host memory "
                                               "(PAPER.md L835-838 'query response time')"}
         # comparators on the same batch (same timing protocol, fewer steps)

@@ -165,7 +165,9 @@ enum { PSB_ALGO_PSB = 0, PSB_ALGO_BNB = 1, PSB_ALGO_BRUTE = 2 };
  * traversal counters to `stats`, a DEVICE array int64[q][8]:
  *   {internal-node fetches from memory, leaf scans, point ids loaded,
  *    internal-node visits served by the path cache, leaf scans that changed the
- *    kNN list, keys merged into the list, 0, 0}.
+ *    kNN list, keys merged into the list, t_start, t_end}
+ * where t_start/t_end are the device %globaltimer (ns) when the warp took the
+ * query and when it finished it: the in-batch service time.
  * The counters define the algorithmic bytes of a launch:
  *   fetches*fanout*2*d*4 + leaf_scans*fanout*d*4 + ids*4 + q*(4*d + 8*k).
  * The traversal (and hence every counter) is deterministic: a counting run and

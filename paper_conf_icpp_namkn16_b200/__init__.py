@@ -196,7 +196,8 @@ def psb_knn_stats(index: Index, queries, k: int, algo: int = PSB_ALGO_PSB, varia
                   stream=None, out=None):
     """psb_knn_ex plus per-query counters: returns (ids, dists, stats int64 [q, 8] on device)
     with stats = {node fetches, leaf scans, id loads, path-cache hits, changing leaf scans,
-    keys merged, 0, 0} (include/psb.h)."""
+    keys merged, t_start ns, t_end ns} (include/psb.h; the last two are the device
+    %globaltimer when the warp took / finished the query)."""
     torch = _torch()
     queries, q, ids, dists = _query_buffers(index, queries, k, out)
     stats = torch.zeros((q, 8), dtype=torch.int64, device=f"cuda:{index.device}")

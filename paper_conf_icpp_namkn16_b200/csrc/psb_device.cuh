@@ -445,9 +445,17 @@ struct TopK {
 // algorithmic bytes of a launch without changing the traversal.
 // Compiled in only for the psb_knn_stats instantiations (ON = true): the timed
 // kernels carry no counting code.
+__device__ __forceinline__ int64_t global_ns()
+{
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return (int64_t)t;
+}
 template <bool ON>
 struct Stats {
     uint32_t fetch = 0, hit = 0, leaf = 0, ids = 0, offers = 0, cand = 0;
+    int64_t t0 = 0;   // %globaltimer at the query's start (in-batch service time)
+    __device__ __forceinline__ Stats() { if (ON) t0 = global_ns(); }
     __device__ __forceinline__ void node(bool fetched) { if (ON) { fetched ? ++fetch : ++hit; } }
     __device__ __forceinline__ void scan() { if (ON) ++leaf; }
     __device__ __forceinline__ void id_loads(int n) { if (ON) ids += n; }
@@ -462,8 +470,8 @@ struct Stats {
             o[3] = hit;     // internal visits served by the path cache
             o[4] = offers;  // leaf scans that changed the kNN list
             o[5] = cand;    // keys merged into the kNN list
-            o[6] = 0;
-            o[7] = 0;
+            o[6] = t0;            // %globaltimer (ns) when the warp took the query
+            o[7] = global_ns();   // ... and when it finished it (before the row store)
         }
     }
 };

@@ -328,15 +328,17 @@ def test_host_buffers_and_stats(c2):
             torch.cuda.synchronize()
             assert_same((i.cpu().numpy(), dd.cpu().numpy()), e, f"stats algo={algo} var={var}")
             st = st.cpu().numpy()
+            assert (st[:, 7] >= st[:, 6]).all() and (st[:, 6] > 0).all()   # service-time stamps
+            st = st[:, :6]
             assert (st[:, 1] >= 1).all()                 # every query scans a leaf
             assert (st[:, 0] >= idx.levels).all()        # and fetches at least one root-to-leaf path
             got.append(st)
         i2, _, st2 = psb.psb_knn_stats(idx, qd, cfg.k, algo=algo)
         torch.cuda.synchronize()
-        assert np.array_equal(st2.cpu().numpy(), got[0])          # deterministic
+        assert np.array_equal(st2.cpu().numpy()[:, :6], got[0])          # deterministic
         _, _, st3 = psb.psb_knn_stats(idx, qd, cfg.k, algo=algo, variant=psb.PSB_VAR_LEAF_ORDER)
         torch.cuda.synchronize()
-        assert np.array_equal(st3.cpu().numpy(), got[0])          # same traversal in any query order
+        assert np.array_equal(st3.cpu().numpy()[:, :6], got[0])          # same traversal in any query order
         assert (got[1][:, 3] == 0).all()                           # no cache -> no hits
         assert np.array_equal(got[0][:, 0] + got[0][:, 3], got[1][:, 0])  # same visits, cache or not
         assert np.array_equal(got[0][:, 1], got[1][:, 1])          # same leaves scanned
