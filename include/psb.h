@@ -154,9 +154,15 @@ int psb_knn_bruteforce(const psb_index *idx, const float *queries, int64_t q, in
  *                          share them in L1/L2. Rows are still written in input
  *                          order. With neither bit, leaf order is used when
  *                          q >= 1024 and the leaves (points + ids) exceed 64 MiB.
+ * bit 4 PSB_VAR_PREFETCH_NEXT — with every leaf scan, prefetch the right
+ *                          sibling's coordinates into L1 (the next leaf whenever
+ *                          the scan changes the kNN list, Alg. 1 l.41);
+ * bit 5 PSB_VAR_PREFETCH_IDS — with every leaf scan, prefetch the leaf's point
+ *                          ids into L1 (they are loaded lazily, only for points
+ *                          that pass the distance filter).
  * Results are identical for every variant. */
 enum { PSB_VAR_NOCACHE = 1, PSB_VAR_NOMAXDIST = 2, PSB_VAR_INPUT_ORDER = 4,
-       PSB_VAR_LEAF_ORDER = 8 };
+       PSB_VAR_LEAF_ORDER = 8, PSB_VAR_PREFETCH_NEXT = 16, PSB_VAR_PREFETCH_IDS = 32 };
 int psb_knn_ex(const psb_index *idx, const float *queries, int64_t q, int32_t k,
                int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant);
 enum { PSB_ALGO_PSB = 0, PSB_ALGO_BNB = 1, PSB_ALGO_BRUTE = 2 };

@@ -32,6 +32,7 @@ struct WarpState {
     u64 *scratch;        // [32] top-k merge scratch
     u64 *list;           // [k] large-k list (KS == 0 kernels)
     float *qsmem;        // query (D == 0 only)
+    unsigned pf;         // scan_leaf prefetch flags (PF_NEXT, PF_IDS)
 };
 
 __device__ __forceinline__ WarpState warp_state(unsigned char *smem, int H, int F, bool qsmem, int kbig = 0)
@@ -49,6 +50,7 @@ __device__ __forceinline__ WarpState warp_state(unsigned char *smem, int H, int 
     s.list = reinterpret_cast<u64 *>(base + off);
     off += (size_t)kbig * 8;
     s.qsmem = reinterpret_cast<float *>(base + off);
+    s.pf = 0;
     return s;
 }
 
@@ -195,7 +197,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
             const int j = node;
             bool changed = true;                                 // pass-1 leaves: already offered
             if (pass1 || j < pass1_lo || j > pass1_hi)
-                changed = scan_leaf<D, V, KS, ST>(ix, j, q, lane, T, k, thr, S, ws.scratch);
+                changed = scan_leaf<D, V, KS, ST>(ix, j, q, lane, T, k, thr, S, ws.scratch, ws.pf);
             if (pass1) {
                 pass1_hi = j;
                 const int64_t left = ix.n - (int64_t)j * F;
@@ -284,7 +286,7 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
                 ++lvl;
             }
         } else {
-            scan_leaf<D, V, KS, ST>(ix, node, q, lane, T, k, thr, S, ws.scratch);
+            scan_leaf<D, V, KS, ST>(ix, node, q, lane, T, k, thr, S, ws.scratch, ws.pf);
             pd = fminf(pd, key_dist(thr));
             from_c = (int)(node % F);
             node /= F;
@@ -344,7 +346,8 @@ closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, 
     {                                                                                                 \
         extern __shared__ __align__(16) unsigned char smem[];                                         \
         const int lane = threadIdx.x & 31;                                                            \
-        const WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);                 \
+        WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);                       \
+        ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) ? PF_NEXT : 0u) | ((variant & PSB_VAR_PREFETCH_IDS) ? PF_IDS : 0u); \
         const bool use_cache = !(variant & PSB_VAR_NOCACHE);                                          \
         const bool use_max = !(variant & PSB_VAR_NOMAXDIST);                                          \
         int64_t qi = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);                        \
@@ -438,7 +441,7 @@ __device__ __forceinline__ void psb_part_query(const DevIndex &ix, const float *
     int64_t seen = 0;
     while (seen < k && pass1_hi + 1 < hi) {
         ++pass1_hi;
-        scan_leaf<D, V, KS, ST>(ix, pass1_hi, q, lane, T, k, thr, S, ws.scratch);
+        scan_leaf<D, V, KS, ST>(ix, pass1_hi, q, lane, T, k, thr, S, ws.scratch, ws.pf);
         const int64_t left = ix.n - (int64_t)pass1_hi * F;
         seen += left < F ? left : F;
     }
@@ -483,7 +486,7 @@ __device__ __forceinline__ void psb_part_query(const DevIndex &ix, const float *
             if (j >= pass1_lo && j <= pass1_hi) {
                 changed = true;
             } else {
-                changed = scan_leaf<D, V, KS, ST>(ix, j, q, lane, T, k, thr, S, ws.scratch);
+                changed = scan_leaf<D, V, KS, ST>(ix, j, q, lane, T, k, thr, S, ws.scratch, ws.pf);
             }
             pd = fminf(pd, key_dist(thr));
             if (pd < published) { if (lane == 0) publish_pd(g, pd); published = pd; }
@@ -510,7 +513,8 @@ psb_split_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int
     const int lane = threadIdx.x & 31;
     const int64_t w = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
     if (w >= nq * parts) return;
-    const WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);
+    WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);
+    ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) ? PF_NEXT : 0u) | ((variant & PSB_VAR_PREFETCH_IDS) ? PF_IDS : 0u);
     psb_part_query<D, V, KS, ST, SPH>(ix, queries, w / parts, (int)(w % parts), parts, k, part_ids, part_dists, gpd, ws,
                                  !(variant & PSB_VAR_NOCACHE), !(variant & PSB_VAR_NOMAXDIST), lane);
 }

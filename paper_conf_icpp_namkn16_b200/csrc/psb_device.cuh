@@ -23,6 +23,7 @@ typedef unsigned long long u64;
 #define PSB_INSERT_MAX 2   // up to this many candidates are inserted one by one, more are merged
 #endif
 constexpr unsigned FULL = 0xffffffffu;
+enum : unsigned { PF_NEXT = 1u, PF_IDS = 2u };   // scan_leaf prefetch flags
 // (dist, id) packed as one u64 key: for dist >= +0 the IEEE bit pattern orders
 // like the value, so u64 order == lexicographic (dist, id) order for ids >= 0.
 // The pad (+inf, -1) = 0x7F800000FFFFFFFF is larger than every real key.
@@ -558,16 +559,19 @@ struct TopK<0> {
 template <int D, int V, int KS, bool ST>
 __device__ __forceinline__ bool scan_leaf(const DevIndex &ix, int leaf, const Query<D> &q,
                                           int lane, TopK<KS> &T, int k, u64 &thr, Stats<ST> &S,
-                                          u64 *scratch)
+                                          u64 *scratch, unsigned pf)
 {
     constexpr int F = 32 * V;
     float dist[V];
     S.scan();
-#if PSB_PREFETCH_NEXT
-    // speculative: the right sibling is next whenever this scan changes the list
-    if (leaf + 1 < ix.L && lane < ix.d * V)
+    // Latency hiding (PSB_VAR_PREFETCH_*): the right sibling is the
+    // next leaf whenever this scan changes the list (Alg. 1 l.41), and this leaf's
+    // ids are needed as soon as a distance passes the filter: start both L2->L1
+    // transfers now, without holding registers.
+    if ((pf & PF_NEXT) && leaf + 1 < ix.L && lane < ix.d * V)
         asm volatile("prefetch.global.L1 [%0];" ::"l"(ix.pts + ((int64_t)leaf + 1) * ix.d * F + lane * 32));
-#endif
+    if ((pf & PF_IDS) && lane < V)
+        asm volatile("prefetch.global.L1 [%0];" ::"l"(ix.ids + (int64_t)leaf * F + lane * 32));
     leaf_dists<D, V>(ix.pts + (int64_t)leaf * ix.d * F, q, ix.d, lane, dist);
     const float td = key_dist(thr);
     bool any = false;
