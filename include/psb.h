@@ -160,9 +160,16 @@ int psb_knn_bruteforce(const psb_index *idx, const float *queries, int64_t q, in
  * bit 5 PSB_VAR_PREFETCH_IDS — with every leaf scan, prefetch the leaf's point
  *                          ids into L1 (they are loaded lazily, only for points
  *                          that pass the distance filter).
+ * bit 6 PSB_VAR_P1_INDEX_TIE — pass 1's ClosestLeaf descent (R4) breaks
+ *                          MINDIST ties by child index alone. By default a tie
+ *                          goes to the child with the smaller MAXDIST first (a
+ *                          query inside several overlapping boxes descends into
+ *                          the one that hugs it), which tightens the initial
+ *                          pruning distance (R4).
  * Results are identical for every variant. */
 enum { PSB_VAR_NOCACHE = 1, PSB_VAR_NOMAXDIST = 2, PSB_VAR_INPUT_ORDER = 4,
-       PSB_VAR_LEAF_ORDER = 8, PSB_VAR_PREFETCH_NEXT = 16, PSB_VAR_PREFETCH_IDS = 32 };
+       PSB_VAR_LEAF_ORDER = 8, PSB_VAR_PREFETCH_NEXT = 16, PSB_VAR_PREFETCH_IDS = 32,
+       PSB_VAR_P1_INDEX_TIE = 64 };
 int psb_knn_ex(const psb_index *idx, const float *queries, int64_t q, int32_t k,
                int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant);
 enum { PSB_ALGO_PSB = 0, PSB_ALGO_BNB = 1, PSB_ALGO_BRUTE = 2 };

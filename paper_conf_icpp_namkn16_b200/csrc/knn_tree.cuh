@@ -62,7 +62,7 @@ template <int D, int V, bool SPH>
 __device__ __forceinline__ bool internal_md(const DevIndex &ix, int lvl, int node,
                                             const Query<D> &q, int lane, const WarpState &ws,
                                             bool use_cache, bool use_max, int k, float &pd,
-                                            float (&md)[V])
+                                            float (&md)[V], float (&Md)[V])
 {
     constexpr int F = 32 * V;
     float *cm = ws.cache_md + (size_t)lvl * F + lane * V;
@@ -72,7 +72,6 @@ __device__ __forceinline__ bool internal_md(const DevIndex &ix, int lvl, int nod
         return false;
     }
     const float *blk = ix.nodes + ix.level_off[lvl] + (int64_t)node * ix.blk_floats;
-    float Md[V];
     if (use_max) {
         if constexpr (SPH) sphere_bounds<D, V, true>(blk, q, ix.d, lane, md, Md);
         else node_bounds<D, V, true>(blk, q, ix.d, lane, md, Md);
@@ -89,6 +88,36 @@ __device__ __forceinline__ bool internal_md(const DevIndex &ix, int lvl, int nod
         __syncwarp();
     }
     return true;
+}
+
+// Pass-1 child choice (S2, R4): among this node's children c in [c_lo, c_hi),
+// the argmin of (MINDIST, MAXDIST, c). A query inside several overlapping boxes
+// has MINDIST 0 to all of them; the smaller MAXDIST picks the box that hugs it,
+// which makes ClosestLeaf, hence the initial pruning distance, much tighter
+// (profiles/r01_closest_leaf.md). With index_tie the order is (MINDIST, c).
+template <int V>
+__device__ __forceinline__ int closest_child(const float (&md)[V], const float (&Md)[V], int c_lo, int c_hi,
+                                             int lane, bool index_tie)
+{
+    u64 best = ~0ull;
+#pragma unroll
+    for (int t = 0; t < V; ++t) {
+        const int cc = lane * V + t;
+        const u64 kk = index_tie ? make_key(md[t], cc) : ((u64)__float_as_uint(md[t]) << 32) | __float_as_uint(Md[t]);
+        if (cc >= c_lo && cc < c_hi) best = kk < best ? kk : best;
+    }
+    best = warp_min_u64(best);
+    if (index_tie) return (int)(best & 0xffffffffu);
+    unsigned mine = 0;
+#pragma unroll
+    for (int t = 0; t < V; ++t) {
+        const int cc = lane * V + t;
+        const u64 kk = ((u64)__float_as_uint(md[t]) << 32) | __float_as_uint(Md[t]);
+        mine |= (unsigned)(cc >= c_lo && cc < c_hi && kk == best) << t;
+    }
+    const unsigned bal = __ballot_sync(FULL, mine != 0);
+    const int src = __ffs(bal) - 1;
+    return src * V + (__ffs(__shfl_sync(FULL, mine, src)) - 1);
 }
 
 // Last leaf under (lvl, node): min((node+1)*F^lvl, L) - 1. With span clamped at
@@ -138,6 +167,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     // Pass 2 (Alg. 1 l.6-47): leftmost eligible descent, left-to-right leaf scan,
     // parent-link backtrack.
     bool pass1 = true;
+    const bool p1_index_tie = (ws.pf & PF_P1_INDEX_TIE) != 0;
     int lvl = H;
     int node = 0;
     int pass1_lo = 0, pass1_hi = -1;
@@ -145,22 +175,12 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     int visited = -1;                                            // R10
     while (true) {
         if (lvl > 0) {
-            float md[V];
-            S.node(internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
+            float md[V], Md[V];
+            S.node(internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md, Md));
             const int base = node * F;
             int c;
             if (pass1) {
-                const int nb = (int)ix.nlev[lvl - 1];
-                u64 best = ~0ull;
-#pragma unroll
-                for (int t = 0; t < V; ++t) {
-                    const int cc = lane * V + t;
-                    if (base + cc < nb) {
-                        const u64 kk = make_key(md[t], cc);
-                        best = kk < best ? kk : best;
-                    }
-                }
-                c = (int)(warp_min_u64(best) & 0xffffffffu);
+                c = closest_child<V>(md, Md, 0, (int)ix.nlev[lvl - 1] - base, lane, p1_index_tie);
             } else {
                 // S6: eligible(c) = MINDIST <= pd (R5) and unvisited leaves below (R8).
                 // Subtree leaf ranges are contiguous and increasing in c, so
@@ -255,8 +275,8 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
     int from_c = -1;                        // child we returned from, -1 = fresh visit
     while (true) {
         if (lvl > 0) {
-            float md[V];
-            S.node(internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md));
+            float md[V], Md[V];
+            S.node(internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md, Md));
             u64 from_key = 0;
             if (from_c >= 0) {
                 float v = md[0];
@@ -303,7 +323,8 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
 // 1 (Alg. 1 l.3; R4). One warp per query, no cache, no MAXDIST.
 template <int D, int V, bool SPH>
 __global__ void __launch_bounds__(WARPS_PER_CTA * 32)
-closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, uint32_t *__restrict__ leaf_key)
+closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, uint32_t *__restrict__ leaf_key,
+                    bool index_tie)
 {
     __shared__ float qs[WARPS_PER_CTA][D == 0 ? PSB_DMAX : 1];
     constexpr int F = 32 * V;
@@ -316,19 +337,10 @@ closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, 
     for (int lvl = ix.H; lvl > 0; --lvl) {
         const float *blk = ix.nodes + ix.level_off[lvl] + (int64_t)node * ix.blk_floats;
         float md[V], Md[V];
-        if constexpr (SPH) sphere_bounds<D, V, false>(blk, q, ix.d, lane, md, Md);
-        else node_bounds<D, V, false>(blk, q, ix.d, lane, md, Md);
-        const int base = node * F, nb = (int)ix.nlev[lvl - 1];
-        u64 best = ~0ull;
-#pragma unroll
-        for (int t = 0; t < V; ++t) {
-            const int c = lane * V + t;
-            if (base + c < nb) {
-                const u64 kk = make_key(md[t], c);
-                best = kk < best ? kk : best;
-            }
-        }
-        node = base + (int)(warp_min_u64(best) & 0xffffffffu);
+        if constexpr (SPH) sphere_bounds<D, V, true>(blk, q, ix.d, lane, md, Md);
+        else node_bounds<D, V, true>(blk, q, ix.d, lane, md, Md);
+        const int base = node * F;
+        node = base + closest_child<V>(md, Md, 0, (int)ix.nlev[lvl - 1] - base, lane, index_tie);
     }
     if (lane == 0) leaf_key[qi] = (uint32_t)node;
 }
@@ -347,7 +359,8 @@ closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, 
         extern __shared__ __align__(16) unsigned char smem[];                                         \
         const int lane = threadIdx.x & 31;                                                            \
         WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);                       \
-        ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) ? PF_NEXT : 0u) | ((variant & PSB_VAR_PREFETCH_IDS) ? PF_IDS : 0u); \
+        ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) ? PF_NEXT : 0u) | ((variant & PSB_VAR_PREFETCH_IDS) ? PF_IDS : 0u) | \
+                ((variant & PSB_VAR_P1_INDEX_TIE) ? PF_P1_INDEX_TIE : 0u);                                \
         const bool use_cache = !(variant & PSB_VAR_NOCACHE);                                          \
         const bool use_max = !(variant & PSB_VAR_NOMAXDIST);                                          \
         int64_t qi = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);                        \
@@ -419,21 +432,11 @@ __device__ __forceinline__ void psb_part_query(const DevIndex &ix, const float *
     // pass 1 inside the range: greedy descent among children overlapping [lo, hi)
     int lvl = H, node = 0;
     while (lvl > 0) {
-        float md[V];
-        internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
+        float md[V], Md[V];
+        internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md, Md);
         const int base = node * F, sh = (lvl - 1) * LOGF;
         const int c_lo = (lo >> sh) - base, c_hi = min((int)ix.nlev[lvl - 1] - base, ((hi - 1) >> sh) - base + 1);
-        u64 best = ~0ull;
-#pragma unroll
-        for (int t = 0; t < V; ++t) {
-            const int c = lane * V + t;
-            if (c >= c_lo && c < c_hi) {
-                const u64 kk = make_key(md[t], c);
-                best = kk < best ? kk : best;
-            }
-        }
-        best = warp_min_u64(best);
-        node = base + (int)(best & 0xffffffffu);
+        node = base + closest_child<V>(md, Md, c_lo, c_hi, lane, (ws.pf & PF_P1_INDEX_TIE) != 0);
         --lvl;
     }
     const int pass1_lo = node;
@@ -453,9 +456,9 @@ __device__ __forceinline__ void psb_part_query(const DevIndex &ix, const float *
     int visited = lo - 1;
     while (true) {
         if (lvl > 0) {
-            float md[V];
+            float md[V], Md[V];
             const float gp = shared_pd(g);                       // issued early, used below
-            internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md);
+            internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md, Md);
             pd = fminf(pd, gp);
             const int base = node * F, sh = (lvl - 1) * LOGF;
             const int c_end = min(min(F, (int)ix.nlev[lvl - 1] - base), ((hi - 1) >> sh) - base + 1);
@@ -592,8 +595,8 @@ static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int
             return report_cuda(e, "cudaMallocFromPoolAsync (query order)");
         }
         auto ck = ix.sphere ? closest_leaf_kernel<D, V, true> : closest_leaf_kernel<D, V, false>;
-        ck<<<(unsigned)((nq + WARPS_PER_CTA - 1) / WARPS_PER_CTA), WARPS_PER_CTA * 32, 0, st>>>(ix, queries, nq,
-                                                                                               leaf_key);
+        ck<<<(unsigned)((nq + WARPS_PER_CTA - 1) / WARPS_PER_CTA), WARPS_PER_CTA * 32, 0, st>>>(
+            ix, queries, nq, leaf_key, (variant & PSB_VAR_P1_INDEX_TIE) != 0);
         int rc = report_cuda(cudaGetLastError(), "closest-leaf kernel launch");
         if (rc == PSB_OK) rc = sort_query_order(leaf_key, nq, ix.L, order, pool, st);
         cudaFreeAsync(leaf_key, st);

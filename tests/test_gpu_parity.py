@@ -57,7 +57,7 @@ def test_c1_all_queries(c1, algo):
     assert_same(run(idx, qs, cfg.k, algo), exp, f"C1 {algo}")
 
 
-@pytest.mark.parametrize("variant", [1, 2, 3])
+@pytest.mark.parametrize("variant", [1, 2, 3, 16, 32, 64, 65, 66])
 @pytest.mark.parametrize("algo", ["psb", "bnb"])
 def test_c1_variants(c1, algo, variant):
     cfg, pts, qs, idx, exp = c1
@@ -102,6 +102,9 @@ def test_c2_nocache_and_batches(c2):
     cfg, pts, qs, idx, exp = c2
     sl = slice(0, 3000)
     assert_same(run(idx, qs[sl], cfg.k, "psb", 1), (exp[0][sl], exp[1][sl]), "C2 psb nocache")
+    # pass 1 with the index-only ClosestLeaf tie-break, and with the L1 prefetches
+    assert_same(run(idx, qs[sl], cfg.k, "psb", 64), (exp[0][sl], exp[1][sl]), "C2 psb index tie")
+    assert_same(run(idx, qs[sl], cfg.k, "psb", 16 | 32), (exp[0][sl], exp[1][sl]), "C2 psb prefetch")
     # batching/order independence: single queries and a reversed batch
     for i in (0, 17, 4999):
         assert_same(run(idx, qs[i:i + 1], cfg.k), (exp[0][i:i + 1], exp[1][i:i + 1]), "C2 single")

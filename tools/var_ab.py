@@ -17,7 +17,7 @@ def t(fn, reps=10):
         if i >= 2: ts.append(s.elapsed_time(e))
     return statistics.median(ts)
 name, algo = sys.argv[1], {"psb": 0, "bnb": 1}[sys.argv[2]]
-cfg = W.config(name)
+cfg = W.config("C5" if name == "C5W" else name)          # C5W: the whole 512M-point C5 set
 if name == "C5":
     b = pdist.shard_bounds(cfg.n, 8); pts = cfg.points(n=b[1] - b[0], row0=0)
 else:
@@ -30,4 +30,8 @@ for v in sys.argv[3:]:
     out = psb.psb_knn_ex(idx, qd, cfg.k, algo=algo, variant=var)
     same = True if ref is None else all(torch.equal(a, b) for a, b in zip(out, ref))
     ref = ref or out
-    print(f"{name} {sys.argv[2]} var {var:#x}: {t(lambda: psb.psb_knn_ex(idx, qd, cfg.k, algo=algo, variant=var)):.3f} ms same={same}", flush=True)
+    ms = t(lambda: psb.psb_knn_ex(idx, qd, cfg.k, algo=algo, variant=var))
+    _, _, st = psb.psb_knn_stats(idx, qd, cfg.k, algo=algo, variant=var)
+    m = st[:, :6].double().mean(0).tolist()
+    print(f"{name} {sys.argv[2]} var {var:#x}: {ms:.3f} ms same={same}  per query: fetches {m[0]:.1f} "
+          f"leaves {m[1]:.1f} changing {m[4]:.1f} keys merged {m[5]:.1f}", flush=True)
