@@ -166,10 +166,17 @@ int psb_knn_bruteforce(const psb_index *idx, const float *queries, int64_t q, in
  *                          query inside several overlapping boxes descends into
  *                          the one that hugs it), which tightens the initial
  *                          pruning distance (R4).
+ * bit 7 PSB_VAR_KTH_MAXDIST — bound the k-th neighbour distance at each fetched
+ *                          node by the k-th smallest child MAXDIST, as Alg. 1
+ *                          l.13-15 prints it (every child counted as one point).
+ *                          By default, when k <= fanout, the bound is the
+ *                          smallest MAXDIST over children whose subtrees hold
+ *                          >= k points (R3): tighter, and a warp min
+ *                          instead of a radix select.
  * Results are identical for every variant. */
 enum { PSB_VAR_NOCACHE = 1, PSB_VAR_NOMAXDIST = 2, PSB_VAR_INPUT_ORDER = 4,
        PSB_VAR_LEAF_ORDER = 8, PSB_VAR_PREFETCH_NEXT = 16, PSB_VAR_PREFETCH_IDS = 32,
-       PSB_VAR_P1_INDEX_TIE = 64 };
+       PSB_VAR_P1_INDEX_TIE = 64, PSB_VAR_KTH_MAXDIST = 128 };
 int psb_knn_ex(const psb_index *idx, const float *queries, int64_t q, int32_t k,
                int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant);
 enum { PSB_ALGO_PSB = 0, PSB_ALGO_BNB = 1, PSB_ALGO_BRUTE = 2 };

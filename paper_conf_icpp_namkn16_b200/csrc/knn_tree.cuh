@@ -75,7 +75,22 @@ __device__ __forceinline__ bool internal_md(const DevIndex &ix, int lvl, int nod
     if (use_max) {
         if constexpr (SPH) sphere_bounds<D, V, true>(blk, q, ix.d, lane, md, Md);
         else node_bounds<D, V, true>(blk, q, ix.d, lane, md, Md);
-        pd = kth_bound<V>(Md, k, pd);                    // Alg. 1 l.13-15
+        if (k <= ix.F && !(ws.pf & PF_KTH_RULE)) {
+            // Alg. 1 l.13-15 with point counts (R3): every child subtree but the
+            // last holds >= F >= k points, all within its MAXDIST, so the smallest
+            // MAXDIST over children holding >= k points bounds d_k.
+            const int64_t lastc = ix.nlev[lvl - 1] - 1;
+            const bool last_ok = ix.n - lastc * ix.span[lvl - 1] * ix.F >= k;
+            float m = pd;
+#pragma unroll
+            for (int t = 0; t < V; ++t) {
+                const int64_t gc = (int64_t)node * F + lane * V + t;
+                if (gc < lastc || (gc == lastc && last_ok)) m = fminf(m, Md[t]);
+            }
+            pd = warp_min_f(m);
+        } else {
+            pd = kth_bound<V>(Md, k, pd);                // the k-th smallest MAXDIST
+        }
     } else {
         if constexpr (SPH) sphere_bounds<D, V, false>(blk, q, ix.d, lane, md, Md);
         else node_bounds<D, V, false>(blk, q, ix.d, lane, md, Md);
@@ -360,7 +375,8 @@ closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, 
         const int lane = threadIdx.x & 31;                                                            \
         WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);                       \
         ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) ? PF_NEXT : 0u) | ((variant & PSB_VAR_PREFETCH_IDS) ? PF_IDS : 0u) | \
-                ((variant & PSB_VAR_P1_INDEX_TIE) ? PF_P1_INDEX_TIE : 0u);                                \
+                ((variant & PSB_VAR_P1_INDEX_TIE) ? PF_P1_INDEX_TIE : 0u) |                               \
+                ((variant & PSB_VAR_KTH_MAXDIST) ? PF_KTH_RULE : 0u);                                     \
         const bool use_cache = !(variant & PSB_VAR_NOCACHE);                                          \
         const bool use_max = !(variant & PSB_VAR_NOMAXDIST);                                          \
         int64_t qi = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);                        \
@@ -517,7 +533,8 @@ psb_split_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int
     const int64_t w = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
     if (w >= nq * parts) return;
     WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);
-    ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) ? PF_NEXT : 0u) | ((variant & PSB_VAR_PREFETCH_IDS) ? PF_IDS : 0u);
+    ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) ? PF_NEXT : 0u) | ((variant & PSB_VAR_PREFETCH_IDS) ? PF_IDS : 0u) |
+            ((variant & PSB_VAR_P1_INDEX_TIE) ? PF_P1_INDEX_TIE : 0u) | ((variant & PSB_VAR_KTH_MAXDIST) ? PF_KTH_RULE : 0u);
     psb_part_query<D, V, KS, ST, SPH>(ix, queries, w / parts, (int)(w % parts), parts, k, part_ids, part_dists, gpd, ws,
                                  !(variant & PSB_VAR_NOCACHE), !(variant & PSB_VAR_NOMAXDIST), lane);
 }

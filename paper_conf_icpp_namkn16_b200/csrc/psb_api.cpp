@@ -270,7 +270,8 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
     int rc = check_query_args(fn, ix, queries, q, k, out_ids, out_dists);
     if (rc != PSB_OK) return rc;
     if (variant & ~(uint32_t)(PSB_VAR_NOCACHE | PSB_VAR_NOMAXDIST | PSB_VAR_INPUT_ORDER | PSB_VAR_LEAF_ORDER |
-                              PSB_VAR_PREFETCH_NEXT | PSB_VAR_PREFETCH_IDS | PSB_VAR_P1_INDEX_TIE)) {
+                              PSB_VAR_PREFETCH_NEXT | PSB_VAR_PREFETCH_IDS | PSB_VAR_P1_INDEX_TIE |
+                              PSB_VAR_KTH_MAXDIST)) {
         psb_set_error("%s: unknown variant bits 0x%x", fn, variant);
         return PSB_EINVAL;
     }

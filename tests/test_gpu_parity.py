@@ -57,7 +57,7 @@ def test_c1_all_queries(c1, algo):
     assert_same(run(idx, qs, cfg.k, algo), exp, f"C1 {algo}")
 
 
-@pytest.mark.parametrize("variant", [1, 2, 3, 16, 32, 64, 65, 66])
+@pytest.mark.parametrize("variant", [1, 2, 3, 16, 32, 64, 65, 66, 128, 129, 192])
 @pytest.mark.parametrize("algo", ["psb", "bnb"])
 def test_c1_variants(c1, algo, variant):
     cfg, pts, qs, idx, exp = c1
@@ -105,6 +105,9 @@ def test_c2_nocache_and_batches(c2):
     # pass 1 with the index-only ClosestLeaf tie-break, and with the L1 prefetches
     assert_same(run(idx, qs[sl], cfg.k, "psb", 64), (exp[0][sl], exp[1][sl]), "C2 psb index tie")
     assert_same(run(idx, qs[sl], cfg.k, "psb", 16 | 32), (exp[0][sl], exp[1][sl]), "C2 psb prefetch")
+    # the paper's k-th smallest MAXDIST bound instead of the count-aware one
+    assert_same(run(idx, qs[sl], cfg.k, "psb", 128), (exp[0][sl], exp[1][sl]), "C2 psb k-th MAXDIST")
+    assert_same(run(idx, qs[sl], cfg.k, "bnb", 128), (exp[0][sl], exp[1][sl]), "C2 bnb k-th MAXDIST")
     # batching/order independence: single queries and a reversed batch
     for i in (0, 17, 4999):
         assert_same(run(idx, qs[i:i + 1], cfg.k), (exp[0][i:i + 1], exp[1][i:i + 1]), "C2 single")

@@ -26,3 +26,11 @@ print(f"  queries started in the last 5% before drain: {late.sum()}, their leave
       f"longest query: {lv[np.argmax(dur)]} leaves, started at {s[np.argmax(dur)]:.1f} us")
 c = np.corrcoef(lv, dur)[0, 1]
 print(f"  corr(leaf scans, service time) = {c:.3f}; us per leaf (median) {np.median(dur / np.maximum(lv, 1)):.3f}")
+ids, d = psb.psb_knn(idx, qd, cfg.k)
+kd = d[:, -1].cpu().numpy()
+top = np.argsort(-dur)[:10]
+print("  longest queries: service us / leaves / changing / keys merged / node fetches / k-th dist")
+for i in top:
+    print(f"   q{i:6d}: {dur[i]:7.1f} {st[i,1]:6d} {st[i,4]:5d} {st[i,5]:6d} {st[i,0]:5d} {kd[i]:10.2f}")
+print(f"  median: {np.median(dur):7.1f} {np.median(st[:,1]):6.0f} {np.median(st[:,4]):5.0f} {np.median(st[:,5]):6.0f} "
+      f"{np.median(st[:,0]):5.0f} {np.median(kd):10.2f}")
