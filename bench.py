@@ -382,7 +382,8 @@ def main():
             dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
         extras["e2e"] = {"value": units * args.steps / (float(e2e_t.item()) / 1e3), "unit": UNIT,
                          "h2d_bytes_per_step": int(q * idx.d * 4), "d2h_bytes_per_step": int(q * k * 8),
-                         "api": "psb_knn_ex with pinned host buffers (library stages H2D/D2H on the stream)"}
+                         "api": "psb_knn_ex with pinned host buffers (library copies the queries H2D on the stream; "
+                                "the kernel writes each result row straight into the pinned host output)"}
         if args.mode == "data" and world > 1:
             extras["e2e"]["note"] = "local search only (the data-sharded all-gather runs on device buffers)"
         # single-query latency: launch -> results on the host,

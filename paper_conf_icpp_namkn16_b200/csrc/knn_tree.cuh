@@ -112,19 +112,17 @@ __device__ __forceinline__ bool internal_md(const DevIndex &ix, int lvl, int nod
 // (profiles/r01_closest_leaf.md). With index_tie the order is (MINDIST, c).
 template <int V>
 __device__ __forceinline__ int closest_child(const float (&md)[V], const float (&Md)[V], int c_lo, int c_hi,
-                                             int lane, bool index_tie, bool maxdist_only = false)
+                                             int lane, bool index_tie)
 {
     u64 best = ~0ull;
 #pragma unroll
     for (int t = 0; t < V; ++t) {
         const int cc = lane * V + t;
-        const u64 kk = index_tie ? make_key(md[t], cc)
-                                 : (maxdist_only ? make_key(Md[t], cc)
-                                                 : ((u64)__float_as_uint(md[t]) << 32) | __float_as_uint(Md[t]));
+        const u64 kk = index_tie ? make_key(md[t], cc) : ((u64)__float_as_uint(md[t]) << 32) | __float_as_uint(Md[t]);
         if (cc >= c_lo && cc < c_hi) best = kk < best ? kk : best;
     }
     best = warp_min_u64(best);
-    if (index_tie || maxdist_only) return (int)(best & 0xffffffffu);
+    if (index_tie) return (int)(best & 0xffffffffu);
     unsigned mine = 0;
 #pragma unroll
     for (int t = 0; t < V; ++t) {
@@ -197,8 +195,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
             const int base = node * F;
             int c;
             if (pass1) {
-                c = closest_child<V>(md, Md, 0, (int)ix.nlev[lvl - 1] - base, lane, p1_index_tie,
-                                     (ws.pf & PF_P1_MAXDIST_ONLY) != 0);
+                c = closest_child<V>(md, Md, 0, (int)ix.nlev[lvl - 1] - base, lane, p1_index_tie);
             } else {
                 // S6: eligible(c) = MINDIST <= pd (R5) and unvisited leaves below (R8).
                 // Subtree leaf ranges are contiguous and increasing in c, so
@@ -379,8 +376,7 @@ closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, 
         WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);                       \
         ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) ? PF_NEXT : 0u) | ((variant & PSB_VAR_PREFETCH_IDS) ? PF_IDS : 0u) | \
                 ((variant & PSB_VAR_P1_INDEX_TIE) ? PF_P1_INDEX_TIE : 0u) |                               \
-                ((variant & PSB_VAR_KTH_MAXDIST) ? PF_KTH_RULE : 0u) |                                    \
-                ((variant & 256u) ? PF_P1_MAXDIST_ONLY : 0u);                                             \
+                ((variant & PSB_VAR_KTH_MAXDIST) ? PF_KTH_RULE : 0u);                                     \
         const bool use_cache = !(variant & PSB_VAR_NOCACHE);                                          \
         const bool use_max = !(variant & PSB_VAR_NOMAXDIST);                                          \
         int64_t qi = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);                        \

@@ -260,6 +260,18 @@ static bool is_device_ptr(const void *p)
     return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
+// Device address of page-locked (pinned or registered) host memory, mapped into
+// the device's address space; nullptr for pageable memory.
+static void *mapped_host_ptr(void *p)
+{
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    return a.type == cudaMemoryTypeHost ? a.devicePointer : nullptr;
+}
+
 // Launch one algorithm on device buffers; host buffers (pinned or pageable) are
 // staged through stream-ordered device scratch with copies on the same stream.
 static int knn_impl(const char *fn, const psb_index *ix, const float *queries, int64_t q, int32_t k,
@@ -271,7 +283,7 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
     if (rc != PSB_OK) return rc;
     if (variant & ~(uint32_t)(PSB_VAR_NOCACHE | PSB_VAR_NOMAXDIST | PSB_VAR_INPUT_ORDER | PSB_VAR_LEAF_ORDER |
                               PSB_VAR_PREFETCH_NEXT | PSB_VAR_PREFETCH_IDS | PSB_VAR_P1_INDEX_TIE |
-                              PSB_VAR_KTH_MAXDIST | 256u)) {
+                              PSB_VAR_KTH_MAXDIST)) {
         psb_set_error("%s: unknown variant bits 0x%x", fn, variant);
         return PSB_EINVAL;
     }
@@ -301,7 +313,20 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
         }
         dq = tmp;
     }
+    // Pinned host outputs: the kernels store each finished row straight into host
+    // memory (zero-copy, over PCIe/C2C while the batch runs) instead of staging
+    // the whole result for a copy after the last query; pageable ones are staged.
+    bool staged = ho;
     if (ho) {
+        int32_t *mi = is_device_ptr(out_ids) ? out_ids : static_cast<int32_t *>(mapped_host_ptr(out_ids));
+        float *md = is_device_ptr(out_dists) ? out_dists : static_cast<float *>(mapped_host_ptr(out_dists));
+        if (mi && md) {
+            di = mi;
+            dd = md;
+            staged = false;
+        }
+    }
+    if (staged) {
         if ((e = cudaMallocFromPoolAsync((void **)&di, bo, ix->pool, st)) != cudaSuccess ||
             (e = cudaMallocFromPoolAsync((void **)&dd, bo, ix->pool, st)) != cudaSuccess)
             rc = report_cuda(e, fn);
@@ -311,7 +336,7 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
         rc = algo == PSB_ALGO_BRUTE ? psb::launch_brute(v, dq, q, k, di, dd, st, ix->sm_count, ix->pool)
                                     : psb::launch_tree(algo, v, dq, q, k, di, dd, st, variant, stats, ix->pool, parts);
     }
-    if (ho) {
+    if (staged) {
         if (rc == PSB_OK && ((e = cudaMemcpyAsync(out_ids, di, bo, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||
                              (e = cudaMemcpyAsync(out_dists, dd, bo, cudaMemcpyDeviceToHost, st)) != cudaSuccess))
             rc = report_cuda(e, fn);

@@ -23,7 +23,7 @@ typedef unsigned long long u64;
 #define PSB_INSERT_MAX 2   // up to this many candidates are inserted one by one, more are merged
 #endif
 constexpr unsigned FULL = 0xffffffffu;
-enum : unsigned { PF_NEXT = 1u, PF_IDS = 2u, PF_P1_INDEX_TIE = 4u, PF_KTH_RULE = 8u, PF_P1_MAXDIST_ONLY = 16u };   // per-launch traversal flags
+enum : unsigned { PF_NEXT = 1u, PF_IDS = 2u, PF_P1_INDEX_TIE = 4u, PF_KTH_RULE = 8u };   // per-launch traversal flags
 // (dist, id) packed as one u64 key: for dist >= +0 the IEEE bit pattern orders
 // like the value, so u64 order == lexicographic (dist, id) order for ids >= 0.
 // The pad (+inf, -1) = 0x7F800000FFFFFFFF is larger than every real key.
