@@ -149,6 +149,11 @@ struct Query<0> {
 // MBRs of one node block [d][2][F] (Alg. 1 l.9-12, §III).
 //   MINDIST term: lo-q if q<lo, q-hi if q>hi, else 0;  MAXDIST term: max(|q-lo|,|q-hi|)
 // Empty slots (lo=+inf, hi=-inf) give +inf for both.
+//   With a = fl(lo - q) and c = fl(hi - q) (RN keeps the sign of the exact
+//   difference, and fl(q - hi) = -c exactly): MINDIST term = max(a, -c, 0),
+//   MAXDIST term = max(|a|, |c|), bit for bit the case analysis above. For even
+//   V the differences and the squares run as packed FADD2 / FMUL2 pairs over two
+//   children; the running sums stay scalar __fadd_rn (see acc_sq_diff).
 template <int D, int V, bool MAX>
 __device__ __forceinline__ void node_bounds(const float *__restrict__ blk, const Query<D> &q, int d,
                                             int lane, float (&md)[V], float (&Md)[V])
@@ -161,15 +166,36 @@ __device__ __forceinline__ void node_bounds(const float *__restrict__ blk, const
         ldv<V>(blk + (2 * j) * F + lane * V, lo);
         ldv<V>(blk + (2 * j + 1) * F + lane * V, hi);
         const float qj = q[j];
+        if constexpr (V % 2 == 0) {
+            const u64 qq = f2_pack(qj, qj);
 #pragma unroll
-        for (int t = 0; t < V; ++t) {
-            float a = __fsub_rn(lo[t], qj);   // lo - q   (= -(q - lo) exactly)
-            float b = __fsub_rn(qj, hi[t]);   // q - hi
-            float tm = qj < lo[t] ? a : (qj > hi[t] ? b : 0.f);
-            md[t] = __fadd_rn(md[t], __fmul_rn(tm, tm));
-            if (MAX) {
-                float tx = fmaxf(fabsf(a), fabsf(b));
-                Md[t] = __fadd_rn(Md[t], __fmul_rn(tx, tx));
+            for (int t = 0; t < V; t += 2) {
+                float a0, a1, c0, c1;
+                f2_unpack(f2_sub(f2_pack(lo[t], lo[t + 1]), qq), a0, a1);
+                f2_unpack(f2_sub(f2_pack(hi[t], hi[t + 1]), qq), c0, c1);
+                const float m0 = fmaxf(fmaxf(a0, -c0), 0.f), m1 = fmaxf(fmaxf(a1, -c1), 0.f);
+                float s0, s1;
+                f2_unpack(f2_mul(f2_pack(m0, m1), f2_pack(m0, m1)), s0, s1);
+                md[t] = __fadd_rn(md[t], s0);
+                md[t + 1] = __fadd_rn(md[t + 1], s1);
+                if (MAX) {
+                    const float x0 = fmaxf(fabsf(a0), fabsf(c0)), x1 = fmaxf(fabsf(a1), fabsf(c1));
+                    f2_unpack(f2_mul(f2_pack(x0, x1), f2_pack(x0, x1)), s0, s1);
+                    Md[t] = __fadd_rn(Md[t], s0);
+                    Md[t + 1] = __fadd_rn(Md[t + 1], s1);
+                }
+            }
+        } else {
+#pragma unroll
+            for (int t = 0; t < V; ++t) {
+                const float a = __fsub_rn(lo[t], qj);   // lo - q
+                const float c = __fsub_rn(hi[t], qj);   // hi - q  (q - hi = -c exactly)
+                const float tm = fmaxf(fmaxf(a, -c), 0.f);
+                md[t] = __fadd_rn(md[t], __fmul_rn(tm, tm));
+                if (MAX) {
+                    const float tx = fmaxf(fabsf(a), fabsf(c));
+                    Md[t] = __fadd_rn(Md[t], __fmul_rn(tx, tx));
+                }
             }
         }
     });
