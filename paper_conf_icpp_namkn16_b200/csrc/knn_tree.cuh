@@ -203,13 +203,13 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
                 // base + c >= (visited+1) / F^(lvl-1)   (a warp-uniform threshold).
                 const int c_end = min(F, (int)ix.nlev[lvl - 1] - base);
                 const int c_min = visited + 1 < (int)ix.L ? ((visited + 1) >> ((lvl - 1) * LOGF)) - base : F;
-                unsigned mine = 0;
+                // this lane's children lane*V+t with c_min <= c < c_end, as a bit range
+                const int lo_b = min(max(c_min - lane * V, 0), V), hi_b = min(max(c_end - lane * V, 0), V);
+                unsigned mine = ((1u << hi_b) - 1u) & ~((1u << lo_b) - 1u);
+                unsigned under = 0;
 #pragma unroll
-                for (int t = 0; t < V; ++t) {
-                    const int cc = lane * V + t;
-                    const bool e = cc >= c_min && cc < c_end && md[t] <= pd;
-                    mine |= (unsigned)e << t;
-                }
+                for (int t = 0; t < V; ++t) under |= (unsigned)(md[t] <= pd) << t;
+                mine &= under;
                 const unsigned bal = __ballot_sync(FULL, mine != 0);
                 c = F;
                 if (bal) {                                       // leftmost (R6, R7)
