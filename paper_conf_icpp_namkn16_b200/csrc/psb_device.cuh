@@ -71,8 +71,10 @@ __device__ __forceinline__ u64 f2_mul(u64 a, u64 b)
     return r;
 }
 // dist[t] += (p[t] - q)^2 for V points, pairs packed when V is even.
+// first: dimension 0, where fl(+0 + x) = x for the square x >= +0, so the sum
+// starts at the square (no FADD; bit-identical).
 template <int V>
-__device__ __forceinline__ void acc_sq_diff(float (&dist)[V], const float (&p)[V], float qj)
+__device__ __forceinline__ void acc_sq_diff(float (&dist)[V], const float (&p)[V], float qj, bool first = false)
 {
     if constexpr (V % 2 == 0) {
         const u64 qq = f2_pack(qj, qj);
@@ -81,12 +83,15 @@ __device__ __forceinline__ void acc_sq_diff(float (&dist)[V], const float (&p)[V
             const u64 d2 = f2_sub(f2_pack(p[t], p[t + 1]), qq);
             float a, b;
             f2_unpack(f2_mul(d2, d2), a, b);
-            dist[t] = __fadd_rn(dist[t], a);
-            dist[t + 1] = __fadd_rn(dist[t + 1], b);
+            dist[t] = first ? a : __fadd_rn(dist[t], a);
+            dist[t + 1] = first ? b : __fadd_rn(dist[t + 1], b);
         }
     } else {
 #pragma unroll
-        for (int t = 0; t < V; ++t) dist[t] = __fadd_rn(dist[t], sq_diff(p[t], qj));
+        for (int t = 0; t < V; ++t) {
+            const float x = sq_diff(p[t], qj);
+            dist[t] = first ? x : __fadd_rn(dist[t], x);
+        }
     }
 }
 
@@ -176,13 +181,13 @@ __device__ __forceinline__ void node_bounds(const float *__restrict__ blk, const
                 const float m0 = fmaxf(fmaxf(a0, -c0), 0.f), m1 = fmaxf(fmaxf(a1, -c1), 0.f);
                 float s0, s1;
                 f2_unpack(f2_mul(f2_pack(m0, m1), f2_pack(m0, m1)), s0, s1);
-                md[t] = __fadd_rn(md[t], s0);
-                md[t + 1] = __fadd_rn(md[t + 1], s1);
+                md[t] = j == 0 ? s0 : __fadd_rn(md[t], s0);
+                md[t + 1] = j == 0 ? s1 : __fadd_rn(md[t + 1], s1);
                 if (MAX) {
                     const float x0 = fmaxf(fabsf(a0), fabsf(c0)), x1 = fmaxf(fabsf(a1), fabsf(c1));
                     f2_unpack(f2_mul(f2_pack(x0, x1), f2_pack(x0, x1)), s0, s1);
-                    Md[t] = __fadd_rn(Md[t], s0);
-                    Md[t + 1] = __fadd_rn(Md[t + 1], s1);
+                    Md[t] = j == 0 ? s0 : __fadd_rn(Md[t], s0);
+                    Md[t + 1] = j == 0 ? s1 : __fadd_rn(Md[t + 1], s1);
                 }
             }
         } else {
@@ -260,7 +265,7 @@ __device__ __forceinline__ void leaf_dists(const float *__restrict__ lp, const Q
     for_dims<D>(d, [&](int j) {
         float p[V];
         ldv<V>(lp + j * F + lane * V, p);
-        acc_sq_diff<V>(dist, p, q[j]);
+        acc_sq_diff<V>(dist, p, q[j], j == 0);
     });
 }
 
