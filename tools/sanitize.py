@@ -14,6 +14,14 @@ for name, n, q in (("C1", None, 100), ("C2", 100_000, 64)):
     idx = psb.psb_build(pts, cfg.fanout)
     for algo in (0, 1, 2):
         psb.psb_knn_ex(idx, qd, cfg.k, algo=algo)
+    for var in (psb.PSB_VAR_KTH_MAXDIST, psb.PSB_VAR_P1_INDEX_TIE, psb.PSB_VAR_PREFETCH_NEXT | psb.PSB_VAR_PREFETCH_IDS,
+                psb.PSB_VAR_LEAF_ORDER, psb.PSB_VAR_NOCACHE):
+        psb.psb_knn_ex(idx, qd, cfg.k, variant=var)
+    # pinned host outputs: rows stored by the kernels straight into host memory
+    hi = torch.empty((q, cfg.k), dtype=torch.int32, pin_memory=True)
+    hd = torch.empty((q, cfg.k), dtype=torch.float32, pin_memory=True)
+    for algo in (0, 1, 2):
+        psb.psb_knn_ex(idx, qd.cpu().pin_memory(), cfg.k, algo=algo, out=(hi, hd))
     psb.psb_knn_stats(idx, qd, cfg.k, algo=0)
     psb.psb_knn_split(idx, qd[:4], cfg.k, parts=16)
     ids, d = psb.psb_knn(idx, qd, cfg.k)
