@@ -21,9 +21,15 @@ constexpr double REORDER_MIN_BYTES = 64.0 * (1 << 20);
 // Resident CTAs per SM the traversal kernels are compiled for (register cap
 // 65536 / (128 * blocks)): 8 (<= 64 registers) measured best at d <= 8, 6 (<= 80)
 // at d = 16 and for the runtime-d kernels (profiles/r01_occupancy.md).
+#ifndef PSB_MINBLOCKS_SMALL_D
+#define PSB_MINBLOCKS_SMALL_D 8
+#endif
+#ifndef PSB_MINBLOCKS_LARGE_D
+#define PSB_MINBLOCKS_LARGE_D 6
+#endif
 template <int D>
 struct MinBlocks {
-    static constexpr int value = (D == 0 || D >= 16) ? 6 : 8;
+    static constexpr int value = (D == 0 || D >= 16) ? PSB_MINBLOCKS_LARGE_D : PSB_MINBLOCKS_SMALL_D;
 };
 
 struct WarpState {
