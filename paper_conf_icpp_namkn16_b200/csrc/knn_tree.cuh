@@ -85,14 +85,11 @@ __device__ __forceinline__ bool internal_md(const DevIndex &ix, int lvl, int nod
             // Alg. 1 l.13-15 with point counts (R3): every child subtree but the
             // last holds >= F >= k points, all within its MAXDIST, so the smallest
             // MAXDIST over children holding >= k points bounds d_k.
-            const int64_t lastc = ix.nlev[lvl - 1] - 1;
-            const bool last_ok = ix.n - lastc * ix.span[lvl - 1] * ix.F >= k;
+            const int lim = ix.kcnt_lim[lvl] - (node * F + lane * V);
             float m = pd;
 #pragma unroll
-            for (int t = 0; t < V; ++t) {
-                const int64_t gc = (int64_t)node * F + lane * V + t;
-                if (gc < lastc || (gc == lastc && last_ok)) m = fminf(m, Md[t]);
-            }
+            for (int t = 0; t < V; ++t)
+                if (t <= lim) m = fminf(m, Md[t]);
             pd = warp_min_f(m);
         } else {
             pd = kth_bound<V>(Md, k, pd);                // the k-th smallest MAXDIST
@@ -546,12 +543,19 @@ psb_split_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int
 }
 
 template <int D, int V, int KS>
-static int launch_tree_t(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
+static int launch_tree_t(int algo, const DevIndex &ix0, const float *queries, int64_t nq, int k,
                          int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats,
                          cudaMemPool_t pool, int parts)
 {
-    const size_t smem = WARPS_PER_CTA * WarpSmem::bytes(ix.H, 32 * V, D == 0, KS == 0 ? k : 0);
+    const size_t smem = WARPS_PER_CTA * WarpSmem::bytes(ix0.H, 32 * V, D == 0, KS == 0 ? k : 0);
     int64_t blocks = (nq + WARPS_PER_CTA - 1) / WARPS_PER_CTA;
+    // per-launch view: the count-aware MAXDIST bound's child limit per level (R3)
+    DevIndex ix = ix0;
+    for (int l = 1; l <= ix.H; ++l) {
+        const int64_t lastc = ix.nlev[l - 1] - 1;
+        const bool last_ok = ix.n - lastc * ix.span[l - 1] * ix.F >= k;
+        ix.kcnt_lim[l] = (int32_t)(last_ok ? lastc : lastc - 1);
+    }
     // Counting (stats) kernels are instantiated for the generic-d path only: the
     // traversal, hence every counter, does not depend on the d specialisation.
     using Kern = void (*)(DevIndex, const float *, int64_t, int, int32_t *, float *, uint32_t, int64_t *,

@@ -30,6 +30,9 @@ struct DevIndex {
     int32_t sm_count;                   // of the index's device (launch sizing)
     int32_t sphere;                     // 0: MBR node blocks [d][2][F]; 1: sphere blocks [d+1][F]
     int32_t blk_floats;                 // floats per internal node block
+    // per launch (k known): a child (lvl-1, c) of a level-lvl node holds >= k points
+    // iff c <= kcnt_lim[lvl] (every subtree but the level's last holds >= F points)
+    int32_t kcnt_lim[PSB_MAXLVL + 1];
 };
 
 // Level geometry of a packed tree (shared by the host and GPU loaders).
