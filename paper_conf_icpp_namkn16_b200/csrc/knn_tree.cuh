@@ -77,7 +77,9 @@ __device__ __forceinline__ bool internal_md(const DevIndex &ix, int lvl, int nod
         for (int t = 0; t < V; ++t) md[t] = cm[t];
         return false;
     }
-    const float *blk = ix.nodes + ix.level_off[lvl] + (int64_t)node * ix.blk_floats;
+    // block size: compile-time for MBR nodes of a compile-time d
+    const int64_t bf = (D > 0 && !SPH) ? 2 * D * F : ix.blk_floats;
+    const float *blk = ix.nodes + ix.level_off[lvl] + (int64_t)node * bf;
     if (use_max) {
         if constexpr (SPH) sphere_bounds<D, V, true>(blk, q, ix.d, lane, md, Md);
         else node_bounds<D, V, true>(blk, q, ix.d, lane, md, Md);

@@ -610,7 +610,8 @@ __device__ __forceinline__ bool scan_leaf(const DevIndex &ix, int leaf, const Qu
         asm volatile("prefetch.global.L1 [%0];" ::"l"(ix.pts + ((int64_t)leaf + 1) * ix.d * F + lane * 32));
     if ((pf & PF_IDS) && lane < V)
         asm volatile("prefetch.global.L1 [%0];" ::"l"(ix.ids + (int64_t)leaf * F + lane * 32));
-    leaf_dists<D, V>(ix.pts + (int64_t)leaf * ix.d * F, q, ix.d, lane, dist);
+    constexpr int DC = D;   // compile-time d (0: runtime)
+    leaf_dists<D, V>(ix.pts + (int64_t)leaf * (DC > 0 ? DC : ix.d) * F, q, ix.d, lane, dist);
     const float td = key_dist(thr);
     bool any = false;
 #pragma unroll
