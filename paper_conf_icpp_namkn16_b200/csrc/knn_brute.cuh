@@ -59,7 +59,7 @@ brute_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k, 
             float p[V];
             ldv<V>(lp + j * F, p);
 #pragma unroll
-            for (int i = 0; i < QW; ++i) acc_sq_diff<V>(dist[i], p, q[i][j], j == 0);
+            for (int i = 0; i < QW; ++i) acc_sq_diff<V, PackedSum<D>::value>(dist[i], p, q[i][j], j == 0);
         });
         const int32_t *lid = ix.ids + leaf * F + lane * V;
 #pragma unroll

@@ -43,11 +43,16 @@ __device__ __forceinline__ float sq_diff(float a, float b)
     return __fmul_rn(t, t);
 }
 
-// Packed binary32 pairs (sm_100 FADD2 / FMUL2): each half is rounded exactly as
+// Packed binary32 pairs (sm_100 FADD2 / FFMA2): each half is rounded exactly as
 // the scalar op. ptxas 12.9 contracts a mul.rn.f32x2 that feeds an
 // add.rn.f32x2 into FFMA2 even with --fmad=false, which would break the RN
-// contract; so only the difference and the square are packed and the running
-// sums stay scalar __fadd_rn (tests/test_abi_host.py checks the SASS has no FFMA).
+// contract. So the square is written as fma.rn.f32x2(x, x, -0) with the -0 pair
+// read from constant memory, which ptxas cannot fold: RN(x*x + -0) = RN(x*x)
+// bit for bit (x*x >= +0, and +0 + -0 = +0 under RN), and an fma feeding an add
+// cannot be contracted further. The running sums are then packed add.rn.f32x2.
+// tests/test_abi_host.py checks that the only FFMA2 in the SASS are squares
+// (both multiplicands the same register) with a uniform-register (constant) addend.
+static __constant__ u64 c_neg_zero2 = 0x8000000080000000ull;
 __device__ __forceinline__ u64 f2_pack(float a, float b)
 {
     u64 r;
@@ -64,27 +69,61 @@ __device__ __forceinline__ u64 f2_sub(u64 a, u64 b)
     asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
     return r;
 }
+__device__ __forceinline__ u64 f2_add(u64 a, u64 b)
+{
+    u64 r;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+// x*x per half, rounded once (see above)
+__device__ __forceinline__ u64 f2_sq(u64 a)
+{
+    u64 r;
+    asm("fma.rn.f32x2 %0, %1, %1, %2;" : "=l"(r) : "l"(a), "l"(c_neg_zero2));
+    return r;
+}
 __device__ __forceinline__ u64 f2_mul(u64 a, u64 b)
 {
     u64 r;
     asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
     return r;
 }
+// Packed running sums pay off where the kernels are issue bound (d <= 8). At
+// d = 16 (C4, bound by the latency of its longest queries) the scalar sums
+// measured faster (C4 PSB 17.05 -> 18.2 ms with packed sums, profiles/r01_packed_sums.md).
+#ifndef PSB_PACKED_SUM_MAXD
+#define PSB_PACKED_SUM_MAXD 8
+#endif
+template <int D>
+struct PackedSum {
+    static constexpr bool value = D == 0 || D <= PSB_PACKED_SUM_MAXD;
+};
+// s = first ? x*x : s + x*x per half (first: fl(+0 + y) = y for y >= +0);
+// PS: packed FADD2 sum, else FMUL2 square and scalar sums.
+template <bool PS = true>
+__device__ __forceinline__ void f2_acc_sq(float &s0, float &s1, u64 x, bool first)
+{
+    if constexpr (PS) {
+        const u64 y = f2_sq(x);
+        f2_unpack(first ? y : f2_add(f2_pack(s0, s1), y), s0, s1);
+    } else {
+        float a, b;
+        f2_unpack(f2_mul(x, x), a, b);
+        s0 = first ? a : __fadd_rn(s0, a);
+        s1 = first ? b : __fadd_rn(s1, b);
+    }
+}
 // dist[t] += (p[t] - q)^2 for V points, pairs packed when V is even.
 // first: dimension 0, where fl(+0 + x) = x for the square x >= +0, so the sum
 // starts at the square (no FADD; bit-identical).
-template <int V>
+template <int V, bool PS = true>
 __device__ __forceinline__ void acc_sq_diff(float (&dist)[V], const float (&p)[V], float qj, bool first = false)
 {
     if constexpr (V % 2 == 0) {
         const u64 qq = f2_pack(qj, qj);
 #pragma unroll
         for (int t = 0; t < V; t += 2) {
-            const u64 d2 = f2_sub(f2_pack(p[t], p[t + 1]), qq);
-            float a, b;
-            f2_unpack(f2_mul(d2, d2), a, b);
-            dist[t] = first ? a : __fadd_rn(dist[t], a);
-            dist[t + 1] = first ? b : __fadd_rn(dist[t + 1], b);
+            f2_acc_sq<PS>(dist[t], dist[t + 1], f2_sub(f2_pack(p[t], p[t + 1]), qq), first);
         }
     } else {
 #pragma unroll
@@ -158,7 +197,7 @@ struct Query<0> {
 //   difference, and fl(q - hi) = -c exactly): MINDIST term = max(a, -c, 0),
 //   MAXDIST term = max(|a|, |c|), bit for bit the case analysis above. For even
 //   V the differences and the squares run as packed FADD2 / FMUL2 pairs over two
-//   children; the running sums stay scalar __fadd_rn (see acc_sq_diff).
+//   children, the squares as FFMA2 with a -0 addend and the sums as FADD2 (see f2_sq).
 template <int D, int V, bool MAX>
 __device__ __forceinline__ void node_bounds(const float *__restrict__ blk, const Query<D> &q, int d,
                                             int lane, float (&md)[V], float (&Md)[V])
@@ -179,15 +218,10 @@ __device__ __forceinline__ void node_bounds(const float *__restrict__ blk, const
                 f2_unpack(f2_sub(f2_pack(lo[t], lo[t + 1]), qq), a0, a1);
                 f2_unpack(f2_sub(f2_pack(hi[t], hi[t + 1]), qq), c0, c1);
                 const float m0 = fmaxf(fmaxf(a0, -c0), 0.f), m1 = fmaxf(fmaxf(a1, -c1), 0.f);
-                float s0, s1;
-                f2_unpack(f2_mul(f2_pack(m0, m1), f2_pack(m0, m1)), s0, s1);
-                md[t] = j == 0 ? s0 : __fadd_rn(md[t], s0);
-                md[t + 1] = j == 0 ? s1 : __fadd_rn(md[t + 1], s1);
+                f2_acc_sq<PackedSum<D>::value>(md[t], md[t + 1], f2_pack(m0, m1), j == 0);
                 if (MAX) {
                     const float x0 = fmaxf(fabsf(a0), fabsf(c0)), x1 = fmaxf(fabsf(a1), fabsf(c1));
-                    f2_unpack(f2_mul(f2_pack(x0, x1), f2_pack(x0, x1)), s0, s1);
-                    Md[t] = j == 0 ? s0 : __fadd_rn(Md[t], s0);
-                    Md[t + 1] = j == 0 ? s1 : __fadd_rn(Md[t + 1], s1);
+                    f2_acc_sq<PackedSum<D>::value>(Md[t], Md[t + 1], f2_pack(x0, x1), j == 0);
                 }
             }
         } else {
@@ -265,25 +299,25 @@ __device__ __forceinline__ void leaf_dists(const float *__restrict__ lp, const Q
     for_dims<D>(d, [&](int j) {
         float p[V];
         ldv<V>(lp + j * F + lane * V, p);
-        acc_sq_diff<V>(dist, p, q[j], j == 0);
+        acc_sq_diff<V, PackedSum<D>::value>(dist, p, q[j], j == 0);
     });
 }
 
+// Warp minimum of a float v >= +0 (or +inf, never NaN or -0): non-negative
+// binary32 values order like their bit patterns, so one REDUX.MIN on the bits
+// replaces a 5-step shuffle tree.
 __device__ __forceinline__ float warp_min_f(float v)
 {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v = fminf(v, __shfl_xor_sync(FULL, v, o));
-    return v;
+    return __uint_as_float(__reduce_min_sync(FULL, __float_as_uint(v)));
 }
 
+// Warp minimum of a u64 key: the high words first, then the low words among
+// the lanes holding that high word (two REDUX.MIN).
 __device__ __forceinline__ u64 warp_min_u64(u64 v)
 {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        u64 w = __shfl_xor_sync(FULL, v, o);
-        v = w < v ? w : v;
-    }
-    return v;
+    const uint32_t hi = __reduce_min_sync(FULL, (uint32_t)(v >> 32));
+    const uint32_t lo = __reduce_min_sync(FULL, (uint32_t)(v >> 32) == hi ? (uint32_t)v : 0xffffffffu);
+    return ((u64)hi << 32) | lo;
 }
 
 // S5: k-th smallest of the warp's F MAXDIST values if it is below `pd`, else pd

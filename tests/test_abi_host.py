@@ -168,10 +168,14 @@ def test_pack_modes_and_id_base_only_change_layout():
 
 
 def test_sass_has_no_fused_multiply_add(tmp_path):
-    """Bit-exactness guard: no FFMA/FFMA2 anywhere in libpsb.so's sm_100a SASS
+    """Bit-exactness guard: no contracted FFMA/FFMA2 in libpsb.so's sm_100a SASS
     (the distance and the bounds are sub, mul, add each rounded once, R14).
     ptxas contracts mul.f32x2 -> add.f32x2 into FFMA2 even with --fmad=false,
-    so this check is what keeps the packed FADD2/FMUL2 path honest."""
+    so this check is what keeps the packed path honest. The one FFMA2 form
+    allowed is the square x*x + (-0 pair from constant memory), which rounds
+    exactly like the multiply (psb_device.cuh f2_sq): both multiplicands the
+    same register, the addend a uniform register (loaded from the constant
+    bank; a running sum is per-thread and can never be uniform)."""
     import subprocess
     from concurrent.futures import ThreadPoolExecutor
     subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-xelf", "all", psb.LIB_PATH], cwd=tmp_path,
@@ -193,12 +197,39 @@ def test_sass_has_no_fused_multiply_add(tmp_path):
         out = subprocess.run(["/usr/local/cuda/bin/nvdisasm", str(tmp_path / c)], capture_output=True,
                              text=True).stdout
         fused, fn = [], "?"
+        square = re.compile(r"\bFFMA2 R\d+, (R\d+)(?:\.reuse)?\.F32x2\.HI_LO, \1(?:\.reuse)?\.F32x2\.HI_LO, "
+                            r"(U?R\d+)(?:\.reuse)?\.F32x2\.HI_LO ;")
+        dest = re.compile(r"^\s*/\*[0-9a-f]+\*/\s+(?:@!?U?P\w+\s+)?([A-Z0-9_.]+)\s+(U?R)(\d+)\b")
+        copy = re.compile(r"\b(?:IMAD\.U32|IMAD\.MOV\.U32) (U?R\d+), RZ, RZ, (U?R\d+) ;|\bU?MOV (U?R\d+), (U?R\d+) ;")
+        nz = set()   # registers holding a half of the -0 pair of c_neg_zero2 (program order)
         for l in out.splitlines():
             m = re.match(r"\s*\.text\.(\S+):", l)
             if m:
-                fn = m.group(1)
-            elif re.search(r"\bFFMA2?\b|\bDFMA\b", l) and not re.search(r"ELb1EEEv", fn):
-                fused.append((fn, l.strip()))
+                fn, nz = m.group(1), set()
+                continue
+            if re.search(r"\bFFMA2?\b|\bDFMA\b", l) and not re.search(r"ELb1EEEv", fn):
+                # allowed: a square whose addend is the -0 pair read from the
+                # constant bank (possibly copied between registers)
+                sq = square.search(l)
+                ok = False
+                if sq:
+                    p_, i_ = re.match(r"(U?R)(\d+)", sq.group(2)).groups()
+                    ok = sq.group(2) in nz and "%s%d" % (p_, int(i_) + 1) in nz
+                if not ok:
+                    fused.append((fn, l.strip()))
+            d = dest.match(l)
+            if d:
+                r = int(d.group(3))
+                n = 4 if ".128" in d.group(1) else 2 if re.search(r"\.64|\.WIDE|F32x2|^[A-Z]+2 ", d.group(1) + " " + l) else 1
+                regs = ["%s%d" % (d.group(2), r + i) for i in range(n)]
+                if re.search(r"\bLDCU?\.64 U?R\d+, c\[0x3\]\[U?RZ\]", l):
+                    src_nz = True
+                else:
+                    cm = copy.search(l)
+                    src_nz = bool(cm) and (cm.group(2) or cm.group(4)) in nz
+                nz.difference_update(regs)
+                if src_nz:
+                    nz.update(regs)
         return c, ("FADD" in out or "FMUL" in out), fused
 
     with ThreadPoolExecutor(max_workers=os.cpu_count() or 4) as ex:
