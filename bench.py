@@ -360,7 +360,10 @@ def main():
     kern_s = statistics.mean(step_ms) / 1e3
     peak, peak_src = peaks()
     achieved = alg_bytes / kern_s / 1e9
-    traffic = traffic_from_profiles(args.config, args.algo)
+    # profiles/traffic.json key: the one-GPU slab of a data-sharded run is profiled
+    # as its own workload (tools/prof_one.py C5 = slab 0 of 8 -> "C5slab")
+    prof_cfg = args.config + ("slab" if args.mode == "data" and world == 1 and (args.slab or 1) == 8 else "")
+    traffic = traffic_from_profiles(prof_cfg, args.algo)
 
     extras = {}
     if not args.no_extras:
@@ -462,8 +465,8 @@ def main():
                          "frac": achieved / peak, "traffic": traffic, "kernel": kernel,
                          "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src,
                          "avg_launch_ms": kern_s * 1e3,
-                         "issue": issue_roof(args.config, args.algo, kern_s),
-                         "l2": l2_roof(args.config, args.algo, kern_s),
+                         "issue": issue_roof(prof_cfg, args.algo, kern_s),
+                         "l2": l2_roof(prof_cfg, args.algo, kern_s),
                          "counters_per_query": (None if stats_sum is None else
                                                 {"node_fetches": stats_sum[0] / q, "leaf_scans": stats_sum[1] / q,
                                                  "id_loads": stats_sum[2] / q, "cache_hits": stats_sum[3] / q,
