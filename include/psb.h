@@ -176,10 +176,14 @@ int psb_knn_bruteforce(const psb_index *idx, const float *queries, int64_t q, in
  *                          smallest MAXDIST over children whose subtrees hold
  *                          >= k points (R3): tighter, and a warp min
  *                          instead of a radix select.
+ * bit 8 PSB_VAR_NO_AUTO_PREFETCH — PSB at compile-time d = 16 turns both
+ *                          prefetches (bits 4 and 5) on by default (measured
+ *                          faster there, slower at d <= 8); this
+ *                          bit keeps them off unless bits 4/5 ask for them.
  * Results are identical for every variant. */
 enum { PSB_VAR_NOCACHE = 1, PSB_VAR_NOMAXDIST = 2, PSB_VAR_INPUT_ORDER = 4,
        PSB_VAR_LEAF_ORDER = 8, PSB_VAR_PREFETCH_NEXT = 16, PSB_VAR_PREFETCH_IDS = 32,
-       PSB_VAR_P1_INDEX_TIE = 64, PSB_VAR_KTH_MAXDIST = 128 };
+       PSB_VAR_P1_INDEX_TIE = 64, PSB_VAR_KTH_MAXDIST = 128, PSB_VAR_NO_AUTO_PREFETCH = 256 };
 int psb_knn_ex(const psb_index *idx, const float *queries, int64_t q, int32_t k,
                int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant);
 enum { PSB_ALGO_PSB = 0, PSB_ALGO_BNB = 1, PSB_ALGO_BRUTE = 2 };

@@ -29,6 +29,7 @@ PSB_ALGO_PSB, PSB_ALGO_BNB, PSB_ALGO_BRUTE = 0, 1, 2
 PSB_VAR_NOCACHE, PSB_VAR_NOMAXDIST, PSB_VAR_INPUT_ORDER, PSB_VAR_LEAF_ORDER = 1, 2, 4, 8
 PSB_VAR_PREFETCH_NEXT, PSB_VAR_PREFETCH_IDS, PSB_VAR_P1_INDEX_TIE = 16, 32, 64
 PSB_VAR_KTH_MAXDIST = 128
+PSB_VAR_NO_AUTO_PREFETCH = 256
 PSB_KMAX, PSB_DMAX, PSB_MAX_PARTS = 2048, 64, 16
 FANOUTS = (32, 64, 128, 256, 512)
 

@@ -27,6 +27,15 @@ constexpr double REORDER_MIN_BYTES = 64.0 * (1 << 20);
 #ifndef PSB_MINBLOCKS_LARGE_D
 #define PSB_MINBLOCKS_LARGE_D 6
 #endif
+// PSB prefetches the right sibling's coordinates and the scanned leaf's ids by
+// default at compile-time d >= this (PSB_VAR_NO_AUTO_PREFETCH turns it off): the
+// 8 KB leaf blocks of d = 16 make the long queries that end a C4 batch
+// load-latency bound (C4 16.9 -> 15.9 ms), while at d <= 8 the traversal is
+// issue bound and a prefetch is a wasted L1 fill (C3 6.59 -> 7.08 ms with it;
+// profiles/r01_prefetch.md).
+#ifndef PSB_AUTO_PREFETCH_MIN_D
+#define PSB_AUTO_PREFETCH_MIN_D 16
+#endif
 template <int D>
 struct MinBlocks {
     static constexpr int value = (D == 0 || D >= 16) ? PSB_MINBLOCKS_LARGE_D : PSB_MINBLOCKS_SMALL_D;
@@ -368,7 +377,7 @@ closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, 
 // One warp per query. With `queue` non-null the grid is persistent (as many
 // CTAs as fit on the GPU) and each warp takes the next query from an atomic
 // counter when it finishes one, so a long query never holds an idle block.
-#define PSB_TREE_KERNEL(NAME, BODY)                                                                  \
+#define PSB_TREE_KERNEL(NAME, BODY, AUTO_PF)                                                         \
     template <int D, int V, int KS, bool ST, bool SPH>                                                \
     __global__ void __launch_bounds__(WARPS_PER_CTA * 32, MinBlocks<D>::value)                       \
     NAME(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,                          \
@@ -379,7 +388,9 @@ closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, 
         extern __shared__ __align__(16) unsigned char smem[];                                         \
         const int lane = threadIdx.x & 31;                                                            \
         WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);                       \
-        ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) ? PF_NEXT : 0u) | ((variant & PSB_VAR_PREFETCH_IDS) ? PF_IDS : 0u) | \
+        const bool auto_pf = AUTO_PF && D >= PSB_AUTO_PREFETCH_MIN_D && !(variant & PSB_VAR_NO_AUTO_PREFETCH);  \
+        ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) || auto_pf ? PF_NEXT : 0u) |                          \
+                ((variant & PSB_VAR_PREFETCH_IDS) || auto_pf ? PF_IDS : 0u) |                            \
                 ((variant & PSB_VAR_P1_INDEX_TIE) ? PF_P1_INDEX_TIE : 0u) |                               \
                 ((variant & PSB_VAR_KTH_MAXDIST) ? PF_KTH_RULE : 0u);                                     \
         const bool use_cache = !(variant & PSB_VAR_NOCACHE);                                          \
@@ -398,8 +409,8 @@ closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, 
         }                                                                                             \
     }
 
-PSB_TREE_KERNEL(psb_kernel, psb_query)
-PSB_TREE_KERNEL(bnb_kernel, bnb_query)
+PSB_TREE_KERNEL(psb_kernel, psb_query, true)
+PSB_TREE_KERNEL(bnb_kernel, bnb_query, false)
 
 
 // ---------------------------------------------------------------------------

@@ -283,7 +283,7 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
     if (rc != PSB_OK) return rc;
     if (variant & ~(uint32_t)(PSB_VAR_NOCACHE | PSB_VAR_NOMAXDIST | PSB_VAR_INPUT_ORDER | PSB_VAR_LEAF_ORDER |
                               PSB_VAR_PREFETCH_NEXT | PSB_VAR_PREFETCH_IDS | PSB_VAR_P1_INDEX_TIE |
-                              PSB_VAR_KTH_MAXDIST)) {
+                              PSB_VAR_KTH_MAXDIST | PSB_VAR_NO_AUTO_PREFETCH)) {
         psb_set_error("%s: unknown variant bits 0x%x", fn, variant);
         return PSB_EINVAL;
     }

@@ -57,7 +57,7 @@ def test_c1_all_queries(c1, algo):
     assert_same(run(idx, qs, cfg.k, algo), exp, f"C1 {algo}")
 
 
-@pytest.mark.parametrize("variant", [1, 2, 3, 16, 32, 64, 65, 66, 128, 129, 192])
+@pytest.mark.parametrize("variant", [1, 2, 3, 16, 32, 64, 65, 66, 128, 129, 192, 256, 304])
 @pytest.mark.parametrize("algo", ["psb", "bnb"])
 def test_c1_variants(c1, algo, variant):
     cfg, pts, qs, idx, exp = c1
