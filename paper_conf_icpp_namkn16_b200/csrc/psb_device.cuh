@@ -22,6 +22,12 @@ typedef unsigned long long u64;
 #ifndef PSB_INSERT_MAX
 #define PSB_INSERT_MAX 2   // up to this many candidates are inserted one by one, more are merged
 #endif
+// With a one-segment list (KS = 1, k <= 32) a 32-key merge is cheap enough that
+// only a single candidate is inserted (C5 slab 9.63 -> 9.39 ms, C2/C3 unchanged;
+// C4's two-segment list is faster with 2: profiles/r01ak/ins.txt).
+#ifndef PSB_INSERT_MAX_KS1
+#define PSB_INSERT_MAX_KS1 1
+#endif
 constexpr unsigned FULL = 0xffffffffu;
 enum : unsigned { PF_NEXT = 1u, PF_IDS = 2u, PF_P1_INDEX_TIE = 4u, PF_KTH_RULE = 8u };   // per-launch traversal flags
 // (dist, id) packed as one u64 key: for dist >= +0 the IEEE bit pattern orders
@@ -454,7 +460,7 @@ struct TopK {
             m += __popc(bal[t]);
         }
         if (m == 0) return 0;
-        if (m <= PSB_INSERT_MAX) {
+        if (m <= (KS == 1 ? PSB_INSERT_MAX_KS1 : PSB_INSERT_MAX)) {
             for (int i = 0; i < m; ++i) {                // (t, lane) order; warp-uniform
                 int t0 = 0;                                  // first t with a pending candidate
                 unsigned b = bal[0];
