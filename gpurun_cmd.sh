@@ -1,6 +1,9 @@
-set -x
-O=gpurun_out/r01n; mkdir -p $O
+O=gpurun_out/r01al; mkdir -p $O
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.txt 2>&1; tail -1 $O/smoke.txt
 timeout 1200 python -m pytest tests -m gpu -q -x 2>&1 | tail -3 > $O/pytest_gpu.txt; cat $O/pytest_gpu.txt
-for c in C2 C3 C4 C5 C5W; do timeout 900 python tools/var_ab.py $c psb 0 128 > $O/kth_$c.txt 2>&1; done
-for c in C2 C4; do timeout 900 python tools/var_ab.py $c bnb 0 128 > $O/kth_${c}_bnb.txt 2>&1; done
-cat $O/kth_*
+timeout 600 python tools/var_ab.py C5 psb 0 > $O/cf.txt 2>&1
+timeout 600 python tools/var_ab.py C2 psb 0 >> $O/cf.txt 2>&1
+timeout 900 python bench.py > $O/bench_C2.json 2> $O/bench_C2.err
+timeout 1200 python bench.py --config C5 --mode data --slab 8 > $O/bench_C5slab8.json 2> $O/bench_C5slab8.err
+timeout 1500 python bench.py --config C5 > $O/bench_C5.json 2> $O/bench_C5.err
+cat $O/cf.txt
