@@ -1,17 +1,21 @@
 #!/usr/bin/env python3
 """bench.py — PSB exact kNN throughput on B200 (BASELINE.json metric).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--mode query|data]
-                    [--algo psb|bnb|brute] [--impl ours|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C3] [--mode query|data]
+                    [--algo psb|bnb|brute] [--impl ours|reference] [--weak] [--chunks C]
 
 A step is one pass of the whole hot path (one psb_knn
 launch) over one batch of synthetic queries of the named config, inputs resident
-in HBM. N=1 default workload: BASELINE.json configs[1] (C2: 3-D clustered n=1M,
-fanout 64, 10,000 queries, k=32). Multi-GPU (torchrun, one rank per GPU):
-  --mode query (default): replicated index, each rank answers its own batch of
-      q queries (weak scaling, no collective);
+in HBM. N=1 default workload: BASELINE.json configs[2] (C3: 8-D uniform n=4M,
+fanout 128, 100,000 queries, k=16), the config the metric's "1/2/4/8 B200" is
+quoted on. Multi-GPU (torchrun, one rank per GPU):
+  --mode query (default): replicated index, the fixed batch of q queries is
+      split into N contiguous slices, one per rank, no collective (strong
+      scaling; --weak: every rank answers its own q queries instead);
   --mode data: each rank holds a sub-tree over a slab of the points, every rank
-      answers the same q queries, NCCL all-gather + on-device merge (strong).
+      answers the same q queries, and the per-shard lists are merged from peer
+      memory (psb_exchange, chunked so the exchange overlaps the search) or by
+      NCCL all-gather + on-device merge (--exchange nccl).
 L2 is flushed (256 MiB write) between timed steps; each step is timed with CUDA
 events on the launching stream; the reported time is the max over ranks.
 Prints ONE JSON line on rank 0.
@@ -44,9 +48,15 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=300)
     ap.add_argument("--warmup", type=int, default=10)
-    ap.add_argument("--config", default="C2", choices=sorted(W.CONFIGS))
+    ap.add_argument("--config", default="C3", choices=sorted(W.CONFIGS))
     ap.add_argument("--queries", type=int, default=0, help="override q per step (0 = config's)")
     ap.add_argument("--mode", default="query", choices=["query", "data"])
+    ap.add_argument("--weak", action="store_true",
+                    help="query mode, N>1: every rank answers its own q queries (weak scaling)")
+    ap.add_argument("--chunks", type=int, default=4,
+                    help="data mode, N>1, p2p exchange: query chunks (merge of chunk c overlaps search of c+1)")
+    ap.add_argument("--latency-queries", type=int, default=1000,
+                    help="single-query latency sample (SURVEY §8(d): 1,000 distinct queries)")
     ap.add_argument("--slab", type=int, default=0,
                     help="data mode on ONE GPU: run rank 0's local step of a P-way data-sharded job")
     ap.add_argument("--exchange", default="p2p", choices=["p2p", "nccl"],
@@ -139,7 +149,11 @@ def issue_peak() -> float:
     return 148 * 4 * mhz / 1e3
 
 
-L2_CAP_GBS = 6300 * 1.965   # LTS throughput cap ~6300 B/cycle (B300_MICROARCH.md) at 1965 MHz
+def alu_peak() -> float:
+    """FP32 lane-instruction ceiling, T lane-inst/s: 148 SMs x 4 SMSPs x 32 lanes x
+    1 warp instruction per cycle at the max SM clock (B200_PROFILING.md,
+    MEASURED_PEAKS.json sm_max_mhz); DESIGN.md §6 derives it."""
+    return issue_peak() * 32 / 1e3
 
 
 def cpu_baseline(cfg, pts, qs, k, gpu_ids=None, gpu_d=None) -> dict:
@@ -156,13 +170,20 @@ def cpu_baseline(cfg, pts, qs, k, gpu_ids=None, gpu_d=None) -> dict:
         res = tree.knn(qs, k, threads=threads)
         reps.append(time.perf_counter() - t0)
     bnb_qps = len(qs) / statistics.median(reps)
+    # one thread on a bounded sample (a single-thread number too)
+    n1 = min(len(qs), 2000)
+    t0 = time.perf_counter()
+    tree.knn(qs[:n1], k, threads=1)
+    single_qps = n1 / (time.perf_counter() - t0)
     nb = min(len(qs), 1000 if cfg.n <= 2_000_000 else 100)
     t0 = time.perf_counter()
     bf = oracle.knn_bruteforce(pts, qs[:nb], k, threads=threads)
     bf_qps = nb / (time.perf_counter() - t0)
     out = {"value": bnb_qps, "unit": UNIT, "cores": threads, "kind": "oracle",
            "sample": f"all {len(qs)} queries of {cfg.name} via the oracle's recursive B&B (median of 3; "
-                     f"tree build {t_build:.2f}s excluded); brute-force route on {nb} queries",
+                     f"tree build {t_build:.2f}s excluded); single thread on the first {n1}; "
+                     f"brute-force route on {nb} queries",
+           "single_thread_value": single_qps,
            "bruteforce_value": bf_qps,
            "oracle_routes_agree": bool(np.array_equal(bf[0], res[0][:nb]))}
     if gpu_ids is not None:
@@ -173,7 +194,10 @@ def cpu_baseline(cfg, pts, qs, k, gpu_ids=None, gpu_d=None) -> dict:
 
 # ----------------------------------------------------------------------------- reference arm
 def run_reference(args, rank, world):
-    """--impl reference: the CPU oracle on the host cores (the tier's reference arm)."""
+    """--impl reference: the CPU oracle on the host cores (the tier's reference arm),
+    on this arm's config, metric and unit. Each step is a bounded sample of the
+    workload's query batch (sized from a calibration run so the whole
+    --steps/--warmup run takes about a minute); rank 0 alone runs it."""
     if rank != 0:
         return
     import oracle
@@ -183,32 +207,42 @@ def run_reference(args, rank, world):
     qs = cfg.queries(q)
     tree = oracle.Tree(pts)
     threads = os.cpu_count() or 1
-    for _ in range(max(0, args.warmup)):
-        tree.knn(qs[: min(q, 1000)], cfg.k, threads=threads)
+    t0 = time.perf_counter()
+    tree.knn(qs[: min(q, 1000)], cfg.k, threads=threads)                 # calibration (+ warm-up)
+    per_q = (time.perf_counter() - t0) / min(q, 1000)
+    budget_s = 60.0 / max(1, args.steps + args.warmup)
+    sample = int(max(256, min(q, budget_s / max(per_q, 1e-9))))
+    for i in range(max(0, args.warmup)):
+        o = (i * sample) % q
+        tree.knn(qs[o:o + sample], cfg.k, threads=threads)
     times = []
-    for _ in range(args.steps):
+    done = 0
+    for i in range(args.steps):
+        o = (i * sample) % q
+        batch = qs[o:o + sample]
         t0 = time.perf_counter()
-        tree.knn(qs, cfg.k, threads=threads)
+        tree.knn(batch, cfg.k, threads=threads)
         times.append(time.perf_counter() - t0)
+        done += len(batch)
     total = sum(times)
-    val = q * args.steps / total
+    val = done / total
+    desc = (f"each step: {sample} consecutive queries of the {q}-query {cfg.name} batch (bounded sample) via the "
+            f"oracle's recursive B&B on {threads} host threads")
     line = {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+            "scaling": "weak" if args.weak else "strong", "vs_baseline": None, "dtype": "f32",
             "data": "synthetic (workloads/, seeded)", "impl": "reference",
-            "config": {**cfg.describe(), "q": q, "parallelism": "host threads"},
-            "cpu_baseline": {"value": val, "unit": UNIT, "cores": threads, "kind": "oracle",
-                             "sample": f"each step: all {q} queries of {cfg.name} via the oracle's "
-                                       f"recursive B&B on {threads} host threads"},
+            "config": {**cfg.describe(), "q": q, "parallelism": "host threads (rank 0 only)"},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": desc},
             "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
 # ----------------------------------------------------------------------------- our arm
 def issue_roof(config, algo, kern_s):
-    """Secondary roofline: the traversal kernels are bound by instruction issue once the
-    index sits in L2. ncu's warp-instruction count per launch (same
-    command, committed) over the live mean launch time, against the issue ceiling."""
+    """Instruction issue: ncu's warp-instruction count per launch (same kernel,
+    committed profiles/traffic.json) over the live mean launch time, against the
+    issue ceiling."""
     inst = traffic_from_profiles(config, algo, "warp_inst_per_launch")
     if not inst:
         return None
@@ -217,13 +251,50 @@ def issue_roof(config, algo, kern_s):
             "warp_inst_per_launch": inst, "source": "profiles/traffic.json (ncu smsp__inst_executed.sum)"}
 
 
-def l2_roof(config, algo, kern_s):
-    b = traffic_from_profiles(config, algo, "l2_bytes_per_launch")
-    if not b:
-        return None
-    a = b / kern_s / 1e9
-    return {"achieved": a, "peak": L2_CAP_GBS, "unit": "GB/s", "frac": a / L2_CAP_GBS, "l2_bytes_per_launch": b,
-            "peak_source": "B300_MICROARCH.md LTS cap ~6300 B/cycle x 1965 MHz (guide figure, not measured here)"}
+def roofline(algo, idx, q, k, alg_bytes, kern_s, prof_cfg, l2_peak):
+    """The dominant kernel against the ceilings that can bind it.
+
+    Tree traversals: their algorithmic bytes (every node and leaf block each
+    query touches, counted per query) are served from L1/L2, not DRAM, at every
+    config but the cold first touch, so the primary roofline is those bytes over
+    the launch time against the L2 read bandwidth MEASURED in this run
+    (psb_probe_l2_read). Next to it: DRAM bytes (ncu dram__bytes, committed
+    profiles/traffic.json) against the measured HBM peak, ncu's L2 bytes against
+    the same L2 peak, and warp instructions against the issue ceiling. Brute
+    force: bound by FP32 arithmetic, 1.5 lane-instructions per point-dimension
+    (packed subtract / square / add pairs) against the lane-instruction ceiling."""
+    hbm, hbm_src = peaks()
+    if algo == "brute":
+        ops = 1.5 * idx.n * q * idx.d
+        a = ops / kern_s / 1e12
+        prim = {"bound": "alu", "achieved": a, "peak": alu_peak(), "unit": "T lane-inst/s", "frac": a / alu_peak(),
+                "algorithmic_lane_inst_per_launch": ops,
+                "peak_source": "148 SMs x 4 SMSPs x 32 lanes x 1 inst/cycle x sm_max_mhz (DESIGN.md §6)"}
+    else:
+        a = alg_bytes / kern_s / 1e9
+        prim = {"bound": "l2", "achieved": a, "peak": l2_peak, "unit": "GB/s", "frac": a / l2_peak,
+                "algorithmic_bytes_per_launch": alg_bytes,
+                "peak_source": "measured in this run: psb_probe_l2_read (64 MiB L2-resident, ld.global.cg)"}
+    dram = traffic_from_profiles(prof_cfg, algo, "dram_bytes_per_launch")
+    prim["traffic"] = dram
+    prim["avg_launch_ms"] = kern_s * 1e3
+    levels = {}
+    if dram:
+        levels["hbm"] = {"achieved": dram / kern_s / 1e9, "peak": hbm, "unit": "GB/s",
+                         "frac": dram / kern_s / 1e9 / hbm, "dram_bytes_per_launch": dram,
+                         "peak_source": hbm_src, "source": "profiles/traffic.json (ncu dram__bytes read+write)"}
+    l2b = traffic_from_profiles(prof_cfg, algo, "l2_bytes_per_launch")
+    if l2b:
+        levels["l2_ncu"] = {"achieved": l2b / kern_s / 1e9, "peak": l2_peak, "unit": "GB/s",
+                            "frac": l2b / kern_s / 1e9 / l2_peak, "l2_bytes_per_launch": l2b,
+                            "source": "profiles/traffic.json (ncu lts__t_bytes)"}
+    iss = issue_roof(prof_cfg, algo, kern_s)
+    if iss:
+        levels["issue"] = iss
+    prim.update(levels)
+    cands = {prim["bound"]: prim["frac"], **{n: v["frac"] for n, v in levels.items()}}
+    prim["binding"] = max(cands, key=cands.get)
+    return prim
 
 
 def count_launches(step):
@@ -272,11 +343,15 @@ def main():
     q = args.queries or cfg.q
     k = cfg.k
     algo = {"psb": psb.PSB_ALGO_PSB, "bnb": psb.PSB_ALGO_BNB, "brute": psb.PSB_ALGO_BRUTE}[args.algo]
+    weak = args.mode == "query" and args.weak
     if args.mode == "query":
-        # weak scaling: rank r answers its own batch of q queries on a replica
+        # replicated index; strong scaling: rank r answers slice r of the fixed
+        # batch of q queries (weak: its own batch of q)
         pts = cfg.points()
-        all_q = cfg.queries(q * world)
-        qs = all_q[rank * q:(rank + 1) * q]
+        if weak:
+            qs = cfg.queries(q * world)[rank * q:(rank + 1) * q]
+        else:
+            qs = cfg.queries(q)[pdist.query_slice(q, world, rank)]
         idx = psb.psb_build(pts, cfg.fanout)
     else:
         # rank r holds slab r of the points (global ids via id_base); all ranks see all q queries
@@ -285,22 +360,23 @@ def main():
         pts = cfg.points(n=b[rank + 1] - b[rank], row0=b[rank])
         qs = cfg.queries(q)
         idx = psb.psb_build_ex(pts, cfg.fanout, id_base=b[rank])
+    ql = len(qs)                                   # queries this rank searches per step
     stream = torch.cuda.current_stream()
     qd = torch.from_numpy(qs).cuda()
-    out_i = torch.empty((q, k), dtype=torch.int32, device="cuda")
-    out_d = torch.empty((q, k), dtype=torch.float32, device="cuda")
+    out_i = torch.empty((ql, k), dtype=torch.int32, device="cuda")
+    out_d = torch.empty((ql, k), dtype=torch.float32, device="cuda")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 
     # algorithmic bytes of one launch (deterministic traversal counters)
     if algo == psb.PSB_ALGO_BRUTE:
-        alg_bytes = idx.leaves * idx.fanout * (idx.d * 4) * q + q * (4 * idx.d + 8 * k)
+        alg_bytes = idx.leaves * idx.fanout * (idx.d * 4) * ql + ql * (4 * idx.d + 8 * k)
         stats_sum = None
         in_batch = None
     else:
         _, _, st = psb.psb_knn_stats(idx, qd, k, algo=algo, variant=args.variant, out=(out_i, out_d))
         stn = st.cpu().numpy()
         stats_sum = stn[:, :6].sum(0).tolist()
-        alg_bytes = psb.algorithmic_bytes(idx, stats_sum, q, k)
+        alg_bytes = psb.algorithmic_bytes(idx, stats_sum, ql, k)
         # in-batch service time per query (%globaltimer stamps of the counting launch,
         # SURVEY §8(d) latency (b)); the counting kernel is the runtime-d instantiation
         svc = np.sort((stn[:, 7] - stn[:, 6]) / 1e3)
@@ -313,17 +389,21 @@ def main():
 
     def local_knn(qq, kk):
         return psb.psb_knn_ex(idx, qq, kk, algo=algo, variant=args.variant,
-                              out=(out_i, out_d) if qq.shape[0] == q else None)
+                              out=(out_i, out_d) if qq.shape[0] == ql else None)
 
     ex = None
+    chunks = max(1, args.chunks)
     if args.mode == "data" and world > 1 and args.exchange == "p2p":
         ex = pdist.peer_exchange(q, k)
+        rows = sum(r.stop - r.start for r in pdist.chunk_rows(q, world, rank, chunks))
+        merged = (torch.empty((rows, k), dtype=torch.int32, device="cuda"),
+                  torch.empty((rows, k), dtype=torch.float32, device="cuda"))
 
     def step():
         if args.mode == "query" or world == 1:
             local_knn(qd, k)
         elif ex is not None:
-            pdist.data_sharded_knn_p2p(ex, idx, qd, algo=algo, variant=args.variant)
+            pdist.data_sharded_knn_p2p(ex, idx, qd, algo=algo, variant=args.variant, chunks=chunks, out=merged)
         else:
             pdist.data_sharded_knn(local_knn, pdist.device_merge, qd, k)
 
@@ -354,23 +434,27 @@ def main():
     if world > 1:
         dist.all_reduce(total_ms, op=dist.ReduceOp.MAX)
     total_ms = float(total_ms.item())
-    units = q * world if args.mode == "query" else q
+    units = q * world if weak else q
     value = units * args.steps / (total_ms / 1e3)
     ms_per_step = total_ms / args.steps
     kern_s = statistics.mean(step_ms) / 1e3
-    peak, peak_src = peaks()
-    achieved = alg_bytes / kern_s / 1e9
+    l2_peak = psb.psb_probe_l2_read()             # GB/s, this GPU, this run
     # profiles/traffic.json key: the one-GPU slab of a data-sharded run is profiled
     # as its own workload (tools/prof_one.py C5 = slab 0 of 8 -> "C5slab")
     prof_cfg = args.config + ("slab" if args.mode == "data" and world == 1 and (args.slab or 1) == 8 else "")
-    traffic = traffic_from_profiles(prof_cfg, args.algo)
+    roof = roofline(args.algo, idx, ql, k, alg_bytes, kern_s, prof_cfg, l2_peak)
+    roof["kernel"] = {"psb": "psb_kernel", "bnb": "bnb_kernel", "brute": "brute_kernel+merge_kernel"}[args.algo]
+    if stats_sum is not None:
+        roof["counters_per_query"] = {"node_fetches": stats_sum[0] / ql, "leaf_scans": stats_sum[1] / ql,
+                                      "id_loads": stats_sum[2] / ql, "cache_hits": stats_sum[3] / ql,
+                                      "changing_leaf_scans": stats_sum[4] / ql, "keys_merged": stats_sum[5] / ql}
 
     extras = {}
     if not args.no_extras:
         # e2e through the public API with HOST (pinned) buffers: H2D + kernel + D2H each step
         hq = torch.from_numpy(qs).pin_memory()
-        hi = torch.empty((q, k), dtype=torch.int32, pin_memory=True)
-        hd = torch.empty((q, k), dtype=torch.float32, pin_memory=True)
+        hi = torch.empty((ql, k), dtype=torch.int32, pin_memory=True)
+        hd = torch.empty((ql, k), dtype=torch.float32, pin_memory=True)
         e2e_ms = []
         for i in range(max(3, args.warmup) + args.steps):
             flush.fill_(i & 0xFF)
@@ -384,21 +468,21 @@ def main():
         if world > 1:
             dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
         extras["e2e"] = {"value": units * args.steps / (float(e2e_t.item()) / 1e3), "unit": UNIT,
-                         "h2d_bytes_per_step": int(q * idx.d * 4), "d2h_bytes_per_step": int(q * k * 8),
+                         "h2d_bytes_per_step": int(ql * idx.d * 4), "d2h_bytes_per_step": int(ql * k * 8),
                          "api": "psb_knn_ex with pinned host buffers (library copies the queries H2D on the stream; "
                                 "the kernel writes each result row straight into the pinned host output)"}
         if args.mode == "data" and world > 1:
-            extras["e2e"]["note"] = "local search only (the data-sharded all-gather runs on device buffers)"
+            extras["e2e"]["note"] = "local search only (the data-sharded exchange runs on device buffers)"
         # single-query latency: launch -> results on the host,
         # for PSB (one warp), PSB latency mode (query split over many warps), B&B, brute force
         h1i = torch.empty((1, k), dtype=torch.int32, pin_memory=True)
         h1d = torch.empty((1, k), dtype=torch.float32, pin_memory=True)
-        nl = min(q, 200)
+        nl = min(ql, args.latency_queries)
 
         def lat_of(call, n_lat):
             lat = []
             for i in range(n_lat + 5):
-                h1q = hq[i % q:i % q + 1]
+                h1q = hq[i % ql:i % ql + 1]
                 torch.cuda.synchronize()
                 t0 = time.perf_counter()
                 call(h1q)
@@ -422,11 +506,11 @@ def main():
         # comparators on the same batch (same timing protocol, fewer steps)
         comp = {}
         for name, a in (("psb", psb.PSB_ALGO_PSB), ("bnb", psb.PSB_ALGO_BNB), ("brute", psb.PSB_ALGO_BRUTE)):
-            if name == "brute" and idx.n * q > 2e11:
-                comp[name] = {"skipped": f"n*q = {idx.n * q:.2e} pairs (minutes per batch)"}
+            if name == "brute" and idx.n * ql > 2e11:
+                comp[name] = {"skipped": f"n*q = {idx.n * ql:.2e} pairs (minutes per batch)"}
                 continue
             reps = 20 if name != "brute" else 3
-            reps = reps if q * idx.n < 1e12 else 3
+            reps = reps if ql * idx.n < 1e12 else 3
             ts = []
             for i in range(reps + 2):
                 flush.fill_(i & 0xFF)
@@ -437,7 +521,7 @@ def main():
                 torch.cuda.synchronize()
                 if i >= 2:
                     ts.append(s.elapsed_time(e))
-            comp[name] = {"queries_per_s": q / (statistics.median(ts) / 1e3), "ms": statistics.median(ts)}
+            comp[name] = {"queries_per_s": ql / (statistics.median(ts) / 1e3), "ms": statistics.median(ts)}
         extras["comparators_1gpu"] = comp
 
     cpu = None
@@ -447,31 +531,24 @@ def main():
         cpu = cpu_baseline(cfg, pts, qs, k, out_i.cpu().numpy(), out_d.cpu().numpy())
 
     if rank == 0:
-        kernel = {"psb": "psb_kernel", "bnb": "bnb_kernel", "brute": "brute_kernel+merge_kernel"}[args.algo]
+        if args.mode == "query":
+            par = (f"query-sharded x{world} (replicated index; " +
+                   (f"each rank its own {q} queries, weak)" if weak else f"the {q}-query batch split {world} ways)"))
+        elif world > 1:
+            par = (f"data-sharded x{world} (merge from peer memory, psb_exchange, {chunks} chunks)" if ex is not None
+                   else f"data-sharded x{world} (NCCL all-gather + merge)")
+        else:
+            par = f"data-sharded slab 0 of {max(1, args.slab)} (local step only, 1 GPU)"
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": max(3, args.warmup), "ms_per_step": ms_per_step, "higher_is_better": True,
-            "scaling": "weak" if args.mode == "query" else "strong", "vs_baseline": None, "dtype": "f32",
+            "scaling": "weak" if weak else "strong", "vs_baseline": None, "dtype": "f32",
             "data": "synthetic (workloads/: seeded SplitMix64 uniform / 100-cluster Gaussian)",
-            "config": {**cfg.describe(), "q": q, "algo": args.algo, "variant": args.variant,
-                       "parallelism": (f"query-sharded x{world} (replicated index)" if args.mode == "query"
-                                       else ((f"data-sharded x{world} (merge from peer memory, psb_exchange)"
-                                              if ex is not None else f"data-sharded x{world} (NCCL all-gather + merge)")
-                                             if world > 1 else
-                                             f"data-sharded slab 0 of {max(1, args.slab)} (local step only, 1 GPU)")),
+            "config": {**cfg.describe(), "q": q, "q_per_rank": ql, "algo": args.algo,
+                       "variant": args.variant, "parallelism": par,
                        "points_on_this_gpu": int(pts.shape[0]),
                        "l2": "flushed between steps (256 MiB write)", "index_bytes": idx.device_bytes},
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "kernel": kernel,
-                         "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src,
-                         "avg_launch_ms": kern_s * 1e3,
-                         "issue": issue_roof(prof_cfg, args.algo, kern_s),
-                         "l2": l2_roof(prof_cfg, args.algo, kern_s),
-                         "counters_per_query": (None if stats_sum is None else
-                                                {"node_fetches": stats_sum[0] / q, "leaf_scans": stats_sum[1] / q,
-                                                 "id_loads": stats_sum[2] / q, "cache_hits": stats_sum[3] / q,
-                                                 "changing_leaf_scans": stats_sum[4] / q,
-                                                 "keys_merged": stats_sum[5] / q})},
+            "roofline": roof,
             "clocks": clocks,
             "gpu_launches": args.steps * launches_per_step,
             "gpu_launch_names": launch_names,

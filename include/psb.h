@@ -180,10 +180,15 @@ int psb_knn_bruteforce(const psb_index *idx, const float *queries, int64_t q, in
  *                          prefetches (bits 4 and 5) on by default (measured
  *                          faster there, slower at d <= 8); this
  *                          bit keeps them off unless bits 4/5 ask for them.
+ * bit 9 PSB_VAR_GENERIC_D — run the runtime-d instantiation of the kernels even
+ *                          where a compile-time-d one exists (d, fanout) in
+ *                          {(2,32), (3,64), (3,128), (8,128), (16,128)}: the two
+ *                          traverse identically (tests compare their traces).
  * Results are identical for every variant. */
 enum { PSB_VAR_NOCACHE = 1, PSB_VAR_NOMAXDIST = 2, PSB_VAR_INPUT_ORDER = 4,
        PSB_VAR_LEAF_ORDER = 8, PSB_VAR_PREFETCH_NEXT = 16, PSB_VAR_PREFETCH_IDS = 32,
-       PSB_VAR_P1_INDEX_TIE = 64, PSB_VAR_KTH_MAXDIST = 128, PSB_VAR_NO_AUTO_PREFETCH = 256 };
+       PSB_VAR_P1_INDEX_TIE = 64, PSB_VAR_KTH_MAXDIST = 128, PSB_VAR_NO_AUTO_PREFETCH = 256,
+       PSB_VAR_GENERIC_D = 512 };
 int psb_knn_ex(const psb_index *idx, const float *queries, int64_t q, int32_t k,
                int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant);
 enum { PSB_ALGO_PSB = 0, PSB_ALGO_BNB = 1, PSB_ALGO_BRUTE = 2 };
@@ -203,6 +208,27 @@ int psb_knn_stats(const psb_index *idx, const float *queries, int64_t q, int32_t
                   int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant,
                   int64_t *stats);
 
+/* psb_knn_stats plus the traversal trace of every query (tests and
+ * diagnostics: the visit order of Alg. 1, and of the B&B
+ * comparator). trace is a DEVICE int64[q][cap]: step i of query r's walk is
+ * trace[r][i] = node | level << 32 | flags << 40, where level 0 is a leaf (node =
+ * its sequence id) and level >= 1 an internal node visit (node = its index in
+ * the level), in the order the warp took them; flags:
+ *   PSB_TRACE_PASS1   (1)  the step belongs to pass 1 (getInitialPruningDistance);
+ *   PSB_TRACE_CHANGED (2)  leaf scan that changed the kNN list;
+ *   PSB_TRACE_SKIPPED (4)  pass-2 visit of a leaf already scanned in pass 1
+ *                          (not scanned again);
+ *   PSB_TRACE_FETCHED (8)  internal node fetched from memory (else served by
+ *                          the path cache).
+ * trace_len (DEVICE int32[q]) receives each query's number of steps; steps past
+ * cap are counted but not stored. stats may be NULL. 1 <= cap. The counting
+ * kernels run (compile-time-d ones where they exist, PSB_VAR_GENERIC_D for the
+ * generic ones); the traversal and results are those of psb_knn_ex. */
+enum { PSB_TRACE_PASS1 = 1, PSB_TRACE_CHANGED = 2, PSB_TRACE_SKIPPED = 4, PSB_TRACE_FETCHED = 8 };
+int psb_knn_trace(const psb_index *idx, const float *queries, int64_t q, int32_t k,
+                  int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant,
+                  int64_t *stats, int64_t *trace, int32_t cap, int32_t *trace_len);
+
 /* Merge `parts` per-shard result sets ids/dists[parts][q][k] (each row ascending
  * by (dist, id), ids global) into the first k of their union, out[q][k]
  * (data-sharded mode: the step after the all-gather). Device pointers,
@@ -212,35 +238,62 @@ int psb_merge_topk(const int32_t *ids, const float *dists, int32_t parts, int64_
 
 /* ---- Data-sharded exchange over peer memory (north_star) ----
  * The NCCL route (all-gather of every shard's [q][k] lists + psb_merge_topk) is
- * replaced by one kernel per step that pulls only the rows a rank owns directly
- * out of the peers' result buffers (CUDA IPC mappings over NVLink/NVSwitch) and
- * merges them, after a device-side flag barrier: no collective launch, no
- * staging buffer, P-fold less traffic into each rank than an all-gather.
+ * replaced by kernels that pull only the rows a rank owns directly out of the
+ * peers' result buffers (CUDA IPC mappings over NVLink/NVSwitch) and merge them,
+ * after a device-side flag barrier: no collective launch, no staging buffer,
+ * P-fold less traffic into each rank than an all-gather. (The paper itself is
+ * single-GPU, §V-A; the merge is exact because (dist, id) is a total
+ * order and every global id lives in one slab.)
  *
  * Protocol, one object per rank (all ranks: same parts, q, k):
  *   psb_exchange_create(parts, rank, q, k, &x)   allocates on the current device
- *     two [q][k] result buffers (alternating by epoch parity) and parts flag slots;
- *   psb_exchange_handle(x, blob, cap, &used)     blob (IPC handles) to share with
- *     every rank (e.g. torch.distributed all_gather_object);
+ *     two [q][k] result buffers (alternating by epoch parity), parts 64-bit flag
+ *     slots and a status word; 1 <= parts <= PSB_MAX_PARTS, 1 <= q < 2^32,
+ *     1 <= k <= 128;
+ *   psb_exchange_handle(x, blob, cap, &used)     blob (IPC handles + a random
+ *     per-process nonce) to share with every rank (e.g. torch.distributed
+ *     all_gather_object); blob == NULL: only *used is written;
  *   psb_exchange_connect(x, blobs)               maps all ranks' buffers (blobs in
- *     rank order; a blob from the calling process is used without IPC);
- *   each step, with epoch = 1, 2, 3 ...:
- *     psb_exchange_buffers(x, epoch, &ids, &dists)  this rank's result buffers for
- *       the step: run the local psb_knn* into them (ids global via id_base);
- *     psb_exchange_step(x, epoch, row0, rows, out_ids, out_dists, stream)
- *       stream-ordered after the local search: signals every peer, waits (on the
- *       device) until every peer has signalled `epoch`, then writes the merged
- *       first k of rows [row0, row0+rows) of all parts' lists to out[rows][k].
- *   psb_exchange_status(x, &timed_out)           1 if a wait gave up after 10 s
- *     (a peer never signalled; that step's output is undefined).
- * Every rank must call psb_exchange_step for every epoch. k <= 128,
- * parts <= PSB_MAX_PARTS. Synchronous except psb_exchange_step. */
+ *     rank order). A blob from the calling process (same nonce) is used without
+ *     IPC; if it lives on another device, peer access is enabled;
+ *   each step, with epoch = 1, 2, 3 ... (< 2^31):
+ *     psb_exchange_buffers(x, epoch, &ids, &dists)  this rank's [q][k] result
+ *       buffers for the step: run the local psb_knn* into them (global ids);
+ *     psb_exchange_signal(x, epoch, rows_done, stream)  stream-ordered after the
+ *       local search of rows [0, rows_done): publishes (epoch, rows_done) to
+ *       every peer (release, system scope). Rows may be searched and signalled
+ *       in increasing chunks (rows_done increasing within an epoch) so that the
+ *       merge of one chunk overlaps the search of the next;
+ *     psb_exchange_merge(x, epoch, row0, rows, out_ids, out_dists, stream)
+ *       one single-thread wait kernel until every rank (this one included) has
+ *       signalled (epoch, >= max(row0 + rows, 1)), then one warp per row writes
+ *       the merged first k of rows [row0, row0+rows) of all parts' lists to
+ *       out[rows][k] (device pointers). rows may be 0: the wait still runs (it
+ *       is what makes the double buffering safe), nothing is written;
+ *     psb_exchange_step(x, epoch, row0, rows, out...)  = signal(epoch, q) + merge.
+ *   Every rank must signal each epoch (rows_done = q at the latest) and call
+ *   merge at least once per epoch, after its signals. Within one process, issue
+ *   every rank's signal for a chunk before any rank's merge that waits on it
+ *   (a merge's wait must not be queued ahead of a signal it needs: kernels on
+ *   different streams are not guaranteed to run concurrently).
+ * Failure: the wait gives up after the timeout (10 s by default,
+ * psb_exchange_set_timeout) or at once if an earlier wait gave up. The merge
+ * then writes pad rows (-1, +inf), and from the moment the host can see it
+ * (mapped status word, no synchronisation needed) every psb_exchange_* call on
+ * x except psb_exchange_status / psb_exchange_free returns PSB_ECUDA: the
+ * exchange must be freed and recreated. psb_exchange_status reports it
+ * (1 = timed out) for work the device has completed.
+ * Synchronous except psb_exchange_signal / merge / step. */
 #define PSB_MAX_PARTS 16
 typedef struct psb_exchange psb_exchange; /* opaque */
 int psb_exchange_create(int32_t parts, int32_t rank, int64_t q, int32_t k, psb_exchange **out);
+int psb_exchange_set_timeout(psb_exchange *x, int64_t timeout_ns);
 int psb_exchange_handle(const psb_exchange *x, void *blob, int64_t cap, int64_t *used);
 int psb_exchange_connect(psb_exchange *x, const void *const *blobs);
 int psb_exchange_buffers(const psb_exchange *x, int64_t epoch, int32_t **ids, float **dists);
+int psb_exchange_signal(psb_exchange *x, int64_t epoch, int64_t rows_done, void *stream);
+int psb_exchange_merge(psb_exchange *x, int64_t epoch, int64_t row0, int64_t rows, int32_t *out_ids,
+                       float *out_dists, void *stream);
 int psb_exchange_step(psb_exchange *x, int64_t epoch, int64_t row0, int64_t rows, int32_t *out_ids,
                       float *out_dists, void *stream);
 int psb_exchange_status(const psb_exchange *x, int32_t *timed_out);
@@ -266,12 +319,38 @@ int psb_index_info(const psb_index *idx, int64_t *n, int32_t *d, int32_t *fanout
  * and PSB_EINVAL is returned when host_buf is non-NULL. Synchronous. */
 int psb_index_export(const psb_index *idx, void *host_buf, int64_t cap, int64_t *used);
 
+/* Create an index on the current device from a psb_index_export blob (same
+ * layout): replicas (query-sharded mode: build once, broadcast
+ * the flat buffers, import on every rank) and hand-built trees (tests: the
+ * Fig. 2 tree). The blob is validated before anything is uploaded:
+ * level geometry of a packed tree (nodes_per_level[l] = ceil(previous / fanout)
+ * up to a single root), finite coordinates with id >= 0 for points and +inf
+ * with id -1 for pad slots, header n = the number of points, and every box
+ * bounding its leaf's points or its node's child boxes (empty content: lo =
+ * +inf, hi = -inf) — what exactness needs (MINDIST <= dist <= MAXDIST under RN
+ * rounding). Pad slots may sit anywhere; if a leaf other than the
+ * last holds fewer than `fanout` points, the traversals bound the k-th distance
+ * with the printed k-th-MAXDIST rule (Alg. 1 l.13-15) instead of the
+ * count-aware one (R3). Sphere indexes: PSB_EUNSUPPORTED. The blob is copied
+ * (the caller keeps ownership). Synchronous. */
+int psb_index_import(const void *blob, int64_t size, psb_index **out);
+
 /* Host-only bulk load (no CUDA call, no device needed): runs the same packing as
  * psb_build_ex and writes the psb_index_export blob for it into host_buf
  * (same size protocol as psb_index_export). For layout tests on machines without
  * a GPU; a device index built from the same arguments exports identical bytes. */
 int psb_build_host_blob(const float *points, int64_t n, int32_t d, int32_t fanout, int64_t id_base,
                         uint32_t flags, void *host_buf, int64_t cap, int64_t *used);
+
+/* Measurement probe (not part of the query path): the L2 read bandwidth of the
+ * current device, in GB/s, for the roofline bench.py reports (SURVEY.md §8(d):
+ * the traversal's node and leaf blocks are served mostly from L2, so that is the
+ * memory ceiling their algorithmic bytes are compared with). A `bytes` buffer
+ * (>= 1 MiB; 64 MiB fits B200's L2) is read once to make it L2-resident, then
+ * `passes` times per timed launch with 16-byte L2-only (ld.global.cg) loads by
+ * 4 x 512 threads per SM; *gbs = the best of `reps` CUDA-event-timed launches.
+ * Synchronous; allocates and frees its own buffer. */
+int psb_probe_l2_read(int64_t bytes, int32_t passes, int32_t reps, double *gbs);
 
 /* Release the index and its device memory. NULL is a no-op. */
 void psb_free(psb_index *idx);

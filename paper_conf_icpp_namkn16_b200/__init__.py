@@ -30,15 +30,18 @@ PSB_VAR_NOCACHE, PSB_VAR_NOMAXDIST, PSB_VAR_INPUT_ORDER, PSB_VAR_LEAF_ORDER = 1,
 PSB_VAR_PREFETCH_NEXT, PSB_VAR_PREFETCH_IDS, PSB_VAR_P1_INDEX_TIE = 16, 32, 64
 PSB_VAR_KTH_MAXDIST = 128
 PSB_VAR_NO_AUTO_PREFETCH = 256
+PSB_VAR_GENERIC_D = 512
+PSB_TRACE_PASS1, PSB_TRACE_CHANGED, PSB_TRACE_SKIPPED, PSB_TRACE_FETCHED = 1, 2, 4, 8
 PSB_KMAX, PSB_DMAX, PSB_MAX_PARTS = 2048, 64, 16
 FANOUTS = (32, 64, 128, 256, 512)
 
 # every symbol include/psb.h declares (tests check the .so exports all of them)
 EXPORTS = ("psb_build", "psb_build_ex", "psb_knn", "psb_knn_branch_and_bound", "psb_knn_bruteforce",
-           "psb_knn_ex", "psb_knn_stats", "psb_knn_split", "psb_merge_topk", "psb_index_info", "psb_index_export", "psb_build_host_blob",
+           "psb_knn_ex", "psb_knn_stats", "psb_knn_trace", "psb_knn_split", "psb_merge_topk", "psb_index_info", "psb_index_export", "psb_index_import", "psb_build_host_blob",
            "psb_free", "psb_last_error", "psb_version", "psb_exchange_create", "psb_exchange_handle",
-           "psb_exchange_connect", "psb_exchange_buffers", "psb_exchange_step", "psb_exchange_status",
-           "psb_exchange_free")
+           "psb_exchange_connect", "psb_exchange_buffers", "psb_exchange_signal", "psb_exchange_merge",
+           "psb_exchange_step", "psb_exchange_status", "psb_exchange_set_timeout", "psb_exchange_free",
+           "psb_probe_l2_read")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libpsb.so not built at {LIB_PATH}: run __graft_entry__.build() "
@@ -56,18 +59,24 @@ _sig = {
     "psb_knn_ex": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp, _i32, _u32]),
     "psb_knn_split": (ctypes.c_int, [_vp, _vp, _i64, _i32, _i32, _vp, _vp, _vp]),
     "psb_knn_stats": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp, _i32, _u32, _vp]),
+    "psb_knn_trace": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp, _vp, _i32, _u32, _vp, _vp, _i32, _vp]),
     "psb_merge_topk": (ctypes.c_int, [_vp, _vp, _i32, _i64, _i32, _vp, _vp, _vp]),
     "psb_index_info": (ctypes.c_int, [_vp, _P(_i64), _P(_i32), _P(_i32), _P(_i64), _P(_i32), _P(_i64)]),
     "psb_index_export": (ctypes.c_int, [_vp, _vp, _i64, _P(_i64)]),
+    "psb_index_import": (ctypes.c_int, [_vp, _i64, _P(_vp)]),
     "psb_build_host_blob": (ctypes.c_int, [_vp, _i64, _i32, _i32, _i64, _u32, _vp, _i64, _P(_i64)]),
     "psb_free": (None, [_vp]),
     "psb_exchange_create": (ctypes.c_int, [_i32, _i32, _i64, _i32, _P(_vp)]),
     "psb_exchange_handle": (ctypes.c_int, [_vp, _vp, _i64, _P(_i64)]),
     "psb_exchange_connect": (ctypes.c_int, [_vp, _P(_vp)]),
     "psb_exchange_buffers": (ctypes.c_int, [_vp, _i64, _P(_vp), _P(_vp)]),
+    "psb_exchange_signal": (ctypes.c_int, [_vp, _i64, _i64, _vp]),
+    "psb_exchange_merge": (ctypes.c_int, [_vp, _i64, _i64, _i64, _vp, _vp, _vp]),
     "psb_exchange_step": (ctypes.c_int, [_vp, _i64, _i64, _i64, _vp, _vp, _vp]),
+    "psb_exchange_set_timeout": (ctypes.c_int, [_vp, _i64]),
     "psb_exchange_status": (ctypes.c_int, [_vp, _P(_i32)]),
     "psb_exchange_free": (None, [_vp]),
+    "psb_probe_l2_read": (ctypes.c_int, [_i64, _i32, _i32, _P(ctypes.c_double)]),
     "psb_last_error": (ctypes.c_char_p, []),
     "psb_version": (ctypes.c_char_p, []),
 }
@@ -168,6 +177,18 @@ def psb_build(points, fanout: int) -> Index:
     return Index(h)
 
 
+def _check_out(out, q: int, k: int, device):
+    """out = (ids, dists): int32 / float32 [q, k] C-contiguous tensors, on `device`
+    or in host memory."""
+    torch = _torch()
+    ids, dists = out
+    for t, dt, name in ((ids, torch.int32, "ids"), (dists, torch.float32, "dists")):
+        if t.dtype != dt or tuple(t.shape) != (q, k) or not t.is_contiguous():
+            raise ValueError(f"out {name} must be a contiguous {dt} [{q}, {k}] tensor")
+        if t.is_cuda and t.device != device:
+            raise ValueError(f"out {name} is on {t.device}, the index on {device}")
+
+
 def _query_buffers(index: Index, queries, k: int, out):
     """Queries: float32 [q, d] tensor on the index's device, or a CPU tensor
     (pinned for asynchronous copies) — then the library stages it on the stream.
@@ -177,21 +198,42 @@ def _query_buffers(index: Index, queries, k: int, out):
         raise ValueError(f"queries must be a float32 [q, {index.d}] tensor")
     queries = queries.contiguous()
     q = queries.shape[0]
+    dev = torch.device("cuda", index.device)
+    if queries.is_cuda and queries.device != dev:
+        raise ValueError(f"queries are on {queries.device}, the index on {dev}")
     if out is None:
         pin = not queries.is_cuda
         ids = torch.empty((q, k), dtype=torch.int32, device=queries.device, pin_memory=pin)
         dists = torch.empty((q, k), dtype=torch.float32, device=queries.device, pin_memory=pin)
     else:
+        _check_out(out, q, k, dev)
         ids, dists = out
     return queries, q, ids, dists
 
 
+def _host_sync(stream, *tensors):
+    """The C ABI is asynchronous and keeps no reference to its buffers. Host
+    tensors (queries read by a stream-ordered copy, outputs written by the
+    kernels) would otherwise be returned while the device still uses them, and a
+    temporary pinned input could be recycled by torch's caching host allocator:
+    with any host tensor, the call waits for its stream before returning."""
+    if any(not t.is_cuda for t in tensors):
+        torch = _torch()
+        s = stream if stream is not None else torch.cuda.current_stream()
+        if hasattr(s, "synchronize"):
+            s.synchronize()
+        else:
+            torch.cuda.ExternalStream(int(s)).synchronize()
+
+
 def psb_knn_ex(index: Index, queries, k: int, algo: int = PSB_ALGO_PSB, variant: int = 0,
                stream=None, out=None):
-    """Asynchronous on `stream` (default: torch's current stream). Returns (ids, dists)."""
+    """Asynchronous on `stream` (default: torch's current stream) for device
+    tensors; waits for the stream when a tensor is in host memory. Returns (ids, dists)."""
     queries, q, ids, dists = _query_buffers(index, queries, k, out)
     _check(_lib.psb_knn_ex(index.handle, queries.data_ptr(), q, k, ids.data_ptr(), dists.data_ptr(),
                            _stream_handle(stream), algo, variant), "psb_knn_ex")
+    _host_sync(stream, queries, ids, dists)
     return ids, dists
 
 
@@ -206,7 +248,34 @@ def psb_knn_stats(index: Index, queries, k: int, algo: int = PSB_ALGO_PSB, varia
     stats = torch.zeros((q, 8), dtype=torch.int64, device=f"cuda:{index.device}")
     _check(_lib.psb_knn_stats(index.handle, queries.data_ptr(), q, k, ids.data_ptr(), dists.data_ptr(),
                               _stream_handle(stream), algo, variant, stats.data_ptr()), "psb_knn_stats")
+    _host_sync(stream, queries, ids, dists)
     return ids, dists, stats
+
+
+def psb_knn_trace(index: Index, queries, k: int, cap: int = 4096, algo: int = PSB_ALGO_PSB, variant: int = 0,
+                  stream=None, out=None):
+    """psb_knn_stats plus each query's traversal steps (include/psb.h psb_knn_trace).
+    Returns (ids, dists, stats [q, 8], trace int64 [q, cap], trace_len int32 [q]), all
+    on the device; decode with trace_steps()."""
+    torch = _torch()
+    queries, q, ids, dists = _query_buffers(index, queries, k, out)
+    dev = f"cuda:{index.device}"
+    stats = torch.zeros((q, 8), dtype=torch.int64, device=dev)
+    trace = torch.full((q, cap), -1, dtype=torch.int64, device=dev)
+    tlen = torch.zeros((q,), dtype=torch.int32, device=dev)
+    _check(_lib.psb_knn_trace(index.handle, queries.data_ptr(), q, k, ids.data_ptr(), dists.data_ptr(),
+                              _stream_handle(stream), algo, variant, stats.data_ptr(), trace.data_ptr(), cap,
+                              tlen.data_ptr()), "psb_knn_trace")
+    _host_sync(stream, queries, ids, dists)
+    return ids, dists, stats, trace, tlen
+
+
+def trace_steps(row, n: int) -> list[tuple[int, int, int]]:
+    """Decode one query's trace row (first n steps) into (level, node, flags)."""
+    out = []
+    for v in [int(x) for x in row[:n]]:
+        out.append(((v >> 32) & 0xFF, v & 0xFFFFFFFF, (v >> 40) & 0xFF))
+    return out
 
 
 def algorithmic_bytes(index: Index, stats, q: int, k: int) -> int:
@@ -221,6 +290,7 @@ def psb_knn(index: Index, queries, k: int, stream=None, out=None):
     queries, q, ids, dists = _query_buffers(index, queries, k, out)
     _check(_lib.psb_knn(index.handle, queries.data_ptr(), q, k, ids.data_ptr(), dists.data_ptr(),
                         _stream_handle(stream)), "psb_knn")
+    _host_sync(stream, queries, ids, dists)
     return ids, dists
 
 
@@ -229,6 +299,7 @@ def psb_knn_split(index: Index, queries, k: int, parts: int = 0, stream=None, ou
     queries, q, ids, dists = _query_buffers(index, queries, k, out)
     _check(_lib.psb_knn_split(index.handle, queries.data_ptr(), q, k, parts, ids.data_ptr(), dists.data_ptr(),
                               _stream_handle(stream)), "psb_knn_split")
+    _host_sync(stream, queries, ids, dists)
     return ids, dists
 
 
@@ -237,6 +308,7 @@ def psb_knn_branch_and_bound(index: Index, queries, k: int, stream=None, out=Non
     _check(_lib.psb_knn_branch_and_bound(index.handle, queries.data_ptr(), q, k, ids.data_ptr(),
                                          dists.data_ptr(), _stream_handle(stream)),
            "psb_knn_branch_and_bound")
+    _host_sync(stream, queries, ids, dists)
     return ids, dists
 
 
@@ -244,6 +316,7 @@ def psb_knn_bruteforce(index: Index, queries, k: int, stream=None, out=None):
     queries, q, ids, dists = _query_buffers(index, queries, k, out)
     _check(_lib.psb_knn_bruteforce(index.handle, queries.data_ptr(), q, k, ids.data_ptr(),
                                    dists.data_ptr(), _stream_handle(stream)), "psb_knn_bruteforce")
+    _host_sync(stream, queries, ids, dists)
     return ids, dists
 
 
@@ -293,22 +366,55 @@ class Exchange:
                "psb_exchange_buffers")
         return pi.value, pd.value
 
-    def local_knn(self, index: "Index", queries, algo: int = PSB_ALGO_PSB, variant: int = 0, stream=None):
-        """begin() + this rank's local search (all q queries, device buffers) into its buffers."""
+    def local_knn(self, index: "Index", queries, algo: int = PSB_ALGO_PSB, variant: int = 0, stream=None,
+                  rows: slice | None = None):
+        """Local search into this rank's buffers. Without `rows`: begin() (next
+        epoch) + all q queries. With `rows` (a slice of the current epoch's rows,
+        chunked mode): only those queries, written to the same rows."""
         assert queries.is_cuda and queries.shape[0] == self.q
-        pi, pd = self.begin()
-        _check(_lib.psb_knn_ex(index.handle, queries.data_ptr(), self.q, self.k, pi, pd, _stream_handle(stream),
-                               algo, variant), "psb_knn_ex (exchange)")
+        if rows is None:
+            pi, pd = self.begin()
+            r0, r1 = 0, self.q
+        else:
+            pi, pd = _vp(), _vp()
+            _check(_lib.psb_exchange_buffers(self._h, self.epoch, ctypes.byref(pi), ctypes.byref(pd)),
+                   "psb_exchange_buffers")
+            pi, pd = pi.value, pd.value
+            r0, r1 = rows.start, rows.stop
+        if r1 > r0:
+            _check(_lib.psb_knn_ex(index.handle, queries[r0:r1].data_ptr(), r1 - r0, self.k, pi + 4 * r0 * self.k,
+                                   pd + 4 * r0 * self.k, _stream_handle(stream), algo, variant),
+                   "psb_knn_ex (exchange)")
 
-    def step(self, row0: int, rows: int, stream=None, out=None):
-        """Signal the peers, wait for all of them (on the device), merge rows [row0, row0+rows)."""
+    def signal(self, rows_done: int | None = None, stream=None):
+        """Publish that rows [0, rows_done) of this epoch are final (default: all q)."""
+        _check(_lib.psb_exchange_signal(self._h, self.epoch, self.q if rows_done is None else rows_done,
+                                        _stream_handle(stream)), "psb_exchange_signal")
+
+    def _out(self, rows, out):
         torch = _torch()
         if out is None:
-            out = (torch.empty((rows, self.k), dtype=torch.int32, device="cuda"),
-                   torch.empty((rows, self.k), dtype=torch.float32, device="cuda"))
+            return (torch.empty((rows, self.k), dtype=torch.int32, device="cuda"),
+                    torch.empty((rows, self.k), dtype=torch.float32, device="cuda"))
+        _check_out(out, rows, self.k, torch.device("cuda", torch.cuda.current_device()))
+        return out
+
+    def merge(self, row0: int, rows: int, stream=None, out=None):
+        """Wait (on the device) for every rank's signal, merge rows [row0, row0+rows)."""
+        out = self._out(rows, out)
+        _check(_lib.psb_exchange_merge(self._h, self.epoch, row0, rows, out[0].data_ptr(), out[1].data_ptr(),
+                                       _stream_handle(stream)), "psb_exchange_merge")
+        return out
+
+    def step(self, row0: int, rows: int, stream=None, out=None):
+        """signal() for all q rows, then merge(row0, rows) (one call per rank and epoch)."""
+        out = self._out(rows, out)
         _check(_lib.psb_exchange_step(self._h, self.epoch, row0, rows, out[0].data_ptr(), out[1].data_ptr(),
                                       _stream_handle(stream)), "psb_exchange_step")
         return out
+
+    def set_timeout(self, seconds: float):
+        _check(_lib.psb_exchange_set_timeout(self._h, int(seconds * 1e9)), "psb_exchange_set_timeout")
 
     def timed_out(self) -> bool:
         v = _i32()
@@ -359,6 +465,39 @@ def psb_index_export(index: Index) -> dict:
     return _parse_blob(buf)
 
 
+def psb_index_export_raw(index: Index) -> np.ndarray:
+    """The export blob as raw bytes (uint8)."""
+    used = _i64()
+    _check(_lib.psb_index_export(index.handle, None, 0, ctypes.byref(used)), "psb_index_export")
+    buf = np.empty(used.value, dtype=np.uint8)
+    _check(_lib.psb_index_export(index.handle, buf.ctypes.data, used.value, ctypes.byref(used)),
+           "psb_index_export")
+    return buf
+
+
+def psb_index_import(blob) -> Index:
+    """Index on the current device from an export blob (uint8 array / bytes)."""
+    a = np.ascontiguousarray(np.frombuffer(blob, dtype=np.uint8) if isinstance(blob, (bytes, bytearray)) else blob,
+                             dtype=np.uint8)
+    out = ctypes.c_void_p()
+    _check(_lib.psb_index_import(a.ctypes.data, a.size, ctypes.byref(out)), "psb_index_import")
+    return Index(out.value)
+
+
+def make_blob(pts, ids, nodes: dict, n: int, id_base: int = 0) -> np.ndarray:
+    """Assemble an export blob from arrays: pts [L, d, F] float32, ids [L, F] int32,
+    nodes {level: [count, d, 2, F] float32} (psb_index_export layout)."""
+    pts = np.ascontiguousarray(pts, np.float32)
+    ids = np.ascontiguousarray(ids, np.int32)
+    L, d, F = pts.shape
+    H = max(nodes)
+    nlev = np.array([L] + [nodes[l].shape[0] for l in range(1, H + 1)], np.int64)
+    hdr = np.array([n, d, F, L, H, id_base, int(nlev[1:].sum()), 0], np.int64)
+    parts = [hdr.view(np.uint8), nlev.view(np.uint8), pts.reshape(-1).view(np.uint8), ids.reshape(-1).view(np.uint8)]
+    parts += [np.ascontiguousarray(nodes[l], np.float32).reshape(-1).view(np.uint8) for l in range(1, H + 1)]
+    return np.concatenate(parts)
+
+
 def psb_build_host_blob(points, fanout: int, id_base: int = 0, packing: int = PSB_PACK_HILBERT,
                         raw: bool = False):
     """Host-only bulk load (no CUDA): the export blob of the index psb_build_ex would build."""
@@ -370,6 +509,13 @@ def psb_build_host_blob(points, fanout: int, id_base: int = 0, packing: int = PS
     _check(_lib.psb_build_host_blob(a.ctypes.data, a.shape[0], a.shape[1], fanout, id_base, packing,
                                     buf.ctypes.data, used.value, ctypes.byref(used)), "psb_build_host_blob")
     return buf if raw else _parse_blob(buf)
+
+
+def psb_probe_l2_read(nbytes: int = 64 << 20, passes: int = 50, reps: int = 5) -> float:
+    """Measured L2 read bandwidth of the current device, GB/s (include/psb.h)."""
+    g = ctypes.c_double()
+    _check(_lib.psb_probe_l2_read(nbytes, passes, reps, ctypes.byref(g)), "psb_probe_l2_read")
+    return g.value
 
 
 def psb_free(index: Index):

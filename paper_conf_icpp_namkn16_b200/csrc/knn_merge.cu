@@ -140,22 +140,23 @@ int launch_merge(const int32_t *ids, const float *dists, int parts, int64_t nq, 
 #define PSB_SPECIALISED(X) X(2, 1) X(3, 2) X(3, 4) X(8, 4) X(16, 4)
 
 int launch_tree(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool, int parts)
+                float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool, int parts,
+                const TraceOut &tr)
 {
     int rc = PSB_NOT_INSTANTIATED;
     const int V = ix.F / 32;
 #define TRY(DD, VV)                                                                                  \
     if (rc == PSB_NOT_INSTANTIATED && ix.d == DD && V == VV)                                        \
-        rc = launch_tree_ks<DD, VV>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
+        rc = launch_tree_ks<DD, VV>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts, tr);
     PSB_SPECIALISED(TRY)
 #undef TRY
     if (rc == PSB_NOT_INSTANTIATED) {
         switch (V) {
-        case 1: rc = launch_tree_ks<0, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
-        case 2: rc = launch_tree_ks<0, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
-        case 4: rc = launch_tree_ks<0, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
-        case 8: rc = launch_tree_ks<0, 8>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
-        case 16: rc = launch_tree_ks<0, 16>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts); break;
+        case 1: rc = launch_tree_ks<0, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts, tr); break;
+        case 2: rc = launch_tree_ks<0, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts, tr); break;
+        case 4: rc = launch_tree_ks<0, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts, tr); break;
+        case 8: rc = launch_tree_ks<0, 8>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts, tr); break;
+        case 16: rc = launch_tree_ks<0, 16>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts, tr); break;
         default: break;
         }
     }

@@ -48,6 +48,7 @@ struct WarpState {
     u64 *list;           // [k] large-k list (KS == 0 kernels)
     float *qsmem;        // query (D == 0 only)
     unsigned pf;         // scan_leaf prefetch flags (PF_NEXT, PF_IDS)
+    TraceOut tr;         // psb_knn_trace output (counting kernels only)
 };
 
 __device__ __forceinline__ WarpState warp_state(unsigned char *smem, int H, int F, bool qsmem, int kbig = 0)
@@ -66,6 +67,7 @@ __device__ __forceinline__ WarpState warp_state(unsigned char *smem, int H, int 
     off += (size_t)kbig * 8;
     s.qsmem = reinterpret_cast<float *>(base + off);
     s.pf = 0;
+    s.tr = TraceOut{nullptr, nullptr, 0};
     return s;
 }
 
@@ -189,23 +191,31 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     // hit rate (profiles/r01_icache.md).
     //
     // S2: pass 1, getInitialPruningDistance(Q, ClosestLeaf) (Alg. 1 l.3; R4):
-    // greedy descent by (MINDIST, child index) argmin, k-th-MAXDIST bounds on the
-    // way, then ClosestLeaf and its right siblings until k points are seen; their
-    // points go straight into the kNN list (allowed by R4: pass 2 then treats
-    // these leaves as already scanned).
+    // greedy descent by (MINDIST, MAXDIST, child index) argmin, k-th-MAXDIST
+    // bounds on the way, to ClosestLeaf; then ClosestLeaf and the other leaves of
+    // its parent N* in increasing (MINDIST, index) order while their MINDIST is
+    // <= the running pruning distance (at most 32 leaves). N*'s child MINDISTs
+    // were computed on the way down, so choosing them costs no fetch, and the
+    // k-th distance falls fast: the initial bound is close to d_k. Their points
+    // go straight into the kNN list (allowed by R4); pass 2 treats these leaves
+    // as scanned without a change (R25).
     // Pass 2 (Alg. 1 l.6-47): leftmost eligible descent, left-to-right leaf scan,
     // parent-link backtrack.
     bool pass1 = true;
     const bool p1_index_tie = (ws.pf & PF_P1_INDEX_TIE) != 0;
     int lvl = H;
     int node = 0;
-    int pass1_lo = 0, pass1_hi = -1;
-    int64_t seen = 0;
+    // Pass-1 state lives in the path cache's unused level-0 slot (no registers
+    // held across the loop): p1md[c] = MINDIST of N*'s child c, set to -1 once
+    // that leaf is scanned in pass 1; cache_node[0] = N* (level-1 node id).
+    float *const p1md = ws.cache_md;
     int visited = -1;                                            // R10
     while (true) {
         if (lvl > 0) {
             float md[V], Md[V];
-            S.node(internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md, Md));
+            const bool fetched = internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md, Md);
+            S.node(fetched);
+            S.step(ws.tr, qi, lane, lvl, node, (pass1 ? TR_PASS1 : 0u) | (fetched ? TR_FETCHED : 0u));
             const int base = node * F;
             int c;
             if (pass1) {
@@ -234,7 +244,12 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
             }
             if (c < F) {
                 node = base + c;
-                if (--lvl == 0 && pass1) pass1_lo = node;        // ClosestLeaf
+                if (--lvl == 0 && pass1) {                       // ClosestLeaf; keep N*'s MINDISTs
+#pragma unroll
+                    for (int t = 0; t < V; ++t) p1md[lane * V + t] = md[t];
+                    if (lane == 0) ws.cache_node[0] = base >> LOGF;
+                    __syncwarp();
+                }
             } else {                                             // S7 backtrack (R9)
                 if (lvl == H) break;                             // root exhausted (R10)
                 visited = max_leaf(ix, lvl, node);
@@ -244,24 +259,35 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
         } else {
             // S8-S10: leaf j
             const int j = node;
-            bool changed = true;                                 // pass-1 leaves: already offered
-            if (pass1 || j < pass1_lo || j > pass1_hi)
-                changed = scan_leaf<D, V, KS, ST>(ix, j, q, lane, T, k, thr, S, ws.scratch, ws.pf);
+            bool changed = false;
+            // a pass-1 leaf is not scanned again in pass 2 (its points are in the list)
+            const bool pre = !pass1 && (j >> LOGF) == ws.cache_node[0] && p1md[j & (F - 1)] < 0.f;
+            if (!pre) changed = scan_leaf<D, V, KS, ST>(ix, j, q, lane, T, k, thr, S, ws.scratch, ws.pf);
+            S.step(ws.tr, qi, lane, 0, j, (pass1 ? TR_PASS1 : 0u) | (changed ? TR_CHANGED : 0u) | (pre ? TR_SKIPPED : 0u));
+            pd = fminf(pd, key_dist(thr));                       // Alg. 1 l.37
             if (pass1) {
-                pass1_hi = j;
-                const int64_t left = ix.n - (int64_t)j * F;
-                seen += left < F ? left : F;
-                if (seen < k && j + 1 < (int)ix.L) {
-                    node = j + 1;
+                const int b1 = j & ~(F - 1);                     // N*'s first leaf
+                if (lane == 0) p1md[j - b1] = -1.f;              // scanned
+                __syncwarp();
+                // next leaf of N* in (MINDIST, index) order, if its MINDIST <= pd
+                u64 best = ~0ull;
+#pragma unroll
+                for (int t = 0; t < V; ++t) {
+                    const int cc = lane * V + t;
+                    const float v = p1md[cc];
+                    const u64 kk = make_key(v, cc);
+                    if (v >= 0.f && b1 + cc < (int)ix.L && kk < best) best = kk;
+                }
+                best = warp_min_u64(best);
+                if (best != ~0ull && key_dist(best) <= pd) {
+                    node = b1 + (int)(best & 0xffffffffu);
                     continue;
                 }
-                pd = fminf(pd, key_dist(thr));                   // end of pass 1: restart at the root
-                pass1 = false;
+                pass1 = false;                                   // restart at the root
                 lvl = H;
                 node = 0;
                 continue;
             }
-            pd = fminf(pd, key_dist(thr));                       // Alg. 1 l.37
             visited = j;                                         // l.38
             if (j == (int)ix.L - 1) break;                       // R10
             if (changed) {
@@ -274,7 +300,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     }
     // S11
     T.store(k, lane, out_ids + qi * k, out_dists + qi * k);
-    S.write(stats, qi, lane);
+    S.write(stats, ws.tr, qi, lane);
 }
 
 // Stackless B&B: at an internal node take the next child in
@@ -305,7 +331,9 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
     while (true) {
         if (lvl > 0) {
             float md[V], Md[V];
-            S.node(internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md, Md));
+            const bool fetched = internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md, Md);
+            S.node(fetched);
+            S.step(ws.tr, qi, lane, lvl, node, fetched ? TR_FETCHED : 0u);
             u64 from_key = 0;
             if (from_c >= 0) {
                 float v = md[0];
@@ -335,7 +363,8 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
                 ++lvl;
             }
         } else {
-            scan_leaf<D, V, KS, ST>(ix, node, q, lane, T, k, thr, S, ws.scratch, ws.pf);
+            const bool ch = scan_leaf<D, V, KS, ST>(ix, node, q, lane, T, k, thr, S, ws.scratch, ws.pf);
+            S.step(ws.tr, qi, lane, 0, node, ch ? TR_CHANGED : 0u);
             pd = fminf(pd, key_dist(thr));
             from_c = (int)(node % F);
             node /= F;
@@ -343,7 +372,7 @@ __device__ __forceinline__ void bnb_query(const DevIndex &ix, const float *__res
         }
     }
     T.store(k, lane, out_ids + qi * k, out_dists + qi * k);
-    S.write(stats, qi, lane);
+    S.write(stats, ws.tr, qi, lane);
 }
 
 
@@ -383,16 +412,17 @@ closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, 
     NAME(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,                          \
          int32_t *__restrict__ out_ids, float *__restrict__ out_dists, uint32_t variant,             \
          int64_t *__restrict__ stats, unsigned long long *__restrict__ queue,                        \
-         const int32_t *__restrict__ order)                                                           \
+         const int32_t *__restrict__ order, TraceOut tr)                                              \
     {                                                                                                 \
         extern __shared__ __align__(16) unsigned char smem[];                                         \
         const int lane = threadIdx.x & 31;                                                            \
         WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);                       \
+        ws.tr = tr;                                                                                   \
         const bool auto_pf = AUTO_PF && D >= PSB_AUTO_PREFETCH_MIN_D && !(variant & PSB_VAR_NO_AUTO_PREFETCH);  \
         ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) || auto_pf ? PF_NEXT : 0u) |                          \
                 ((variant & PSB_VAR_PREFETCH_IDS) || auto_pf ? PF_IDS : 0u) |                            \
                 ((variant & PSB_VAR_P1_INDEX_TIE) ? PF_P1_INDEX_TIE : 0u) |                               \
-                ((variant & PSB_VAR_KTH_MAXDIST) ? PF_KTH_RULE : 0u);                                     \
+                ((variant & PSB_VAR_KTH_MAXDIST) || ix.irregular ? PF_KTH_RULE : 0u);                     \
         const bool use_cache = !(variant & PSB_VAR_NOCACHE);                                          \
         const bool use_max = !(variant & PSB_VAR_NOMAXDIST);                                          \
         int64_t qi = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);                        \
@@ -550,7 +580,8 @@ psb_split_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int
     if (w >= nq * parts) return;
     WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);
     ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) ? PF_NEXT : 0u) | ((variant & PSB_VAR_PREFETCH_IDS) ? PF_IDS : 0u) |
-            ((variant & PSB_VAR_P1_INDEX_TIE) ? PF_P1_INDEX_TIE : 0u) | ((variant & PSB_VAR_KTH_MAXDIST) ? PF_KTH_RULE : 0u);
+            ((variant & PSB_VAR_P1_INDEX_TIE) ? PF_P1_INDEX_TIE : 0u) |
+            ((variant & PSB_VAR_KTH_MAXDIST) || ix.irregular ? PF_KTH_RULE : 0u);
     psb_part_query<D, V, KS, ST, SPH>(ix, queries, w / parts, (int)(w % parts), parts, k, part_ids, part_dists, gpd, ws,
                                  !(variant & PSB_VAR_NOCACHE), !(variant & PSB_VAR_NOMAXDIST), lane);
 }
@@ -558,7 +589,7 @@ psb_split_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int
 template <int D, int V, int KS>
 static int launch_tree_t(int algo, const DevIndex &ix0, const float *queries, int64_t nq, int k,
                          int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats,
-                         cudaMemPool_t pool, int parts)
+                         cudaMemPool_t pool, int parts, const TraceOut &tr)
 {
     const size_t smem = WARPS_PER_CTA * WarpSmem::bytes(ix0.H, 32 * V, D == 0, KS == 0 ? k : 0);
     int64_t blocks = (nq + WARPS_PER_CTA - 1) / WARPS_PER_CTA;
@@ -569,22 +600,26 @@ static int launch_tree_t(int algo, const DevIndex &ix0, const float *queries, in
         const bool last_ok = ix.n - lastc * ix.span[l - 1] * ix.F >= k;
         ix.kcnt_lim[l] = (int32_t)(last_ok ? lastc : lastc - 1);
     }
-    // Counting (stats) kernels are instantiated for the generic-d path only: the
-    // traversal, hence every counter, does not depend on the d specialisation.
+    // Counting kernels (stats / trace) are instantiated for the generic-d path
+    // and for the compile-time-d MBR kernels, so the counters of a timed
+    // configuration come from the same instantiation as its timed kernel
+    // (PSB_VAR_GENERIC_D selects the generic one; tests compare the two).
+    const bool counting = stats != nullptr || tr.len != nullptr;
     using Kern = void (*)(DevIndex, const float *, int64_t, int, int32_t *, float *, uint32_t, int64_t *,
-                          unsigned long long *, const int32_t *);
+                          unsigned long long *, const int32_t *, TraceOut);
     Kern kern;
     const bool psbk = algo == PSB_ALGO_PSB;
     if constexpr (D == 0) {
         if (ix.sphere)
-            kern = psbk ? (stats ? psb_kernel<D, V, KS, true, true> : psb_kernel<D, V, KS, false, true>)
-                        : (stats ? bnb_kernel<D, V, KS, true, true> : bnb_kernel<D, V, KS, false, true>);
+            kern = psbk ? (counting ? psb_kernel<D, V, KS, true, true> : psb_kernel<D, V, KS, false, true>)
+                        : (counting ? bnb_kernel<D, V, KS, true, true> : bnb_kernel<D, V, KS, false, true>);
         else
-            kern = psbk ? (stats ? psb_kernel<D, V, KS, true, false> : psb_kernel<D, V, KS, false, false>)
-                        : (stats ? bnb_kernel<D, V, KS, true, false> : bnb_kernel<D, V, KS, false, false>);
+            kern = psbk ? (counting ? psb_kernel<D, V, KS, true, false> : psb_kernel<D, V, KS, false, false>)
+                        : (counting ? bnb_kernel<D, V, KS, true, false> : bnb_kernel<D, V, KS, false, false>);
     } else {
-        if (stats) return PSB_NOT_INSTANTIATED;
-        if (ix.sphere) kern = psbk ? psb_kernel<D, V, KS, false, true> : bnb_kernel<D, V, KS, false, true>;
+        if (counting && ix.sphere) return PSB_NOT_INSTANTIATED;
+        if (counting) kern = psbk ? psb_kernel<D, V, KS, true, false> : bnb_kernel<D, V, KS, true, false>;
+        else if (ix.sphere) kern = psbk ? psb_kernel<D, V, KS, false, true> : bnb_kernel<D, V, KS, false, true>;
         else kern = psbk ? psb_kernel<D, V, KS, false, false> : bnb_kernel<D, V, KS, false, false>;
     }
     cudaError_t e;
@@ -592,7 +627,7 @@ static int launch_tree_t(int algo, const DevIndex &ix0, const float *queries, in
         e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return report_cuda(e, "cudaFuncSetAttribute");
     }
-    if (parts > 1 && algo == PSB_ALGO_PSB && !stats && KS != 0) {
+    if (parts > 1 && algo == PSB_ALGO_PSB && !counting && KS != 0) {
         // latency mode: q*parts warps, shared pd per query, then a filtered merge
         auto sk = ix.sphere ? psb_split_kernel<D, V, KS, false, true> : psb_split_kernel<D, V, KS, false, false>;
         if (smem > 48 * 1024) {
@@ -663,7 +698,7 @@ static int launch_tree_t(int algo, const DevIndex &ix0, const float *queries, in
     }
     cudaGetLastError();
     kern<<<(unsigned)blocks, WARPS_PER_CTA * 32, smem, st>>>(ix, queries, nq, k, oi, od, variant, stats, queue,
-                                                             order);
+                                                             order, tr);
     int rc = report_cuda(cudaGetLastError(), "tree kernel launch");
     if (queue) cudaFreeAsync(queue, st);
     if (order) cudaFreeAsync(order, st);
@@ -673,13 +708,14 @@ static int launch_tree_t(int algo, const DevIndex &ix0, const float *queries, in
 template <int D, int V>
 int launch_tree_ks(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k,
                           int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats,
-                         cudaMemPool_t pool, int parts)
+                         cudaMemPool_t pool, int parts, const TraceOut &tr)
 {
-    if (k <= 32) return launch_tree_t<D, V, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
-    if (k <= 64) return launch_tree_t<D, V, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
+    if (D > 0 && (variant & PSB_VAR_GENERIC_D)) return PSB_NOT_INSTANTIATED;
+    if (k <= 32) return launch_tree_t<D, V, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts, tr);
+    if (k <= 64) return launch_tree_t<D, V, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts, tr);
     if constexpr (D == 0) {
-        if (k <= 128) return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);
-        return launch_tree_t<D, V, 0>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts);  // NEXT-3
+        if (k <= 128) return launch_tree_t<D, V, 4>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts, tr);
+        return launch_tree_t<D, V, 0>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts, tr);  // NEXT-3
     }
     return PSB_NOT_INSTANTIATED;   // k > 64: generic-d kernels (keeps compile time down)
 }

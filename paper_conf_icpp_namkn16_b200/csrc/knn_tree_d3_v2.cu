@@ -3,5 +3,6 @@
 
 namespace psb {
 template int launch_tree_ks<3, 2>(int, const DevIndex &, const float *, int64_t, int, int32_t *, float *,
-                                     cudaStream_t, uint32_t, int64_t *, cudaMemPool_t, int);
+                                     cudaStream_t, uint32_t, int64_t *, cudaMemPool_t, int,
+                                     const TraceOut &);
 }

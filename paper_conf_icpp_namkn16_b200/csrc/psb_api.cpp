@@ -2,6 +2,8 @@
 // argument validation, index upload, kernel dispatch, error reporting.
 #include <cuda_runtime.h>
 
+#include <algorithm>
+#include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
@@ -48,6 +50,7 @@ struct psb_index {
     float *nodes = nullptr;
     int64_t device_bytes = 0;
     int32_t sphere = 0, blk_floats = 0;
+    int32_t irregular = 0;          // imported with non-full leaves (DevIndex::irregular)
     cudaMemPool_t pool = nullptr;   // stream-ordered scratch (host-buffer staging, brute-force partials)
 };
 
@@ -89,7 +92,27 @@ static DevIndex dev_view(const psb_index *ix)
     v.sm_count = ix->sm_count;
     v.sphere = ix->sphere;
     v.blk_floats = ix->blk_floats;
+    v.irregular = ix->irregular;
     return v;
+}
+
+// Own pool for per-call scratch; memory stays mapped between calls (a zero
+// release threshold would unmap and remap it at every synchronisation).
+static int make_pool(psb_index *ix, const char *fn)
+{
+    cudaMemPoolProps props;
+    memset(&props, 0, sizeof props);
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = ix->device;
+    cudaError_t e = cudaMemPoolCreate(&ix->pool, &props);
+    if (e != cudaSuccess) {
+        ix->pool = nullptr;
+        return report_cuda(e, fn);
+    }
+    uint64_t keep = UINT64_MAX;
+    cudaMemPoolSetAttribute(ix->pool, cudaMemPoolAttrReleaseThreshold, &keep);
+    return PSB_OK;
 }
 
 extern "C" {
@@ -204,21 +227,10 @@ int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int6
         }
     }
     ix->device_bytes = (int64_t)(bp + bi + bn);
-    // Own pool for per-call scratch; memory stays mapped between calls (a zero
-    // release threshold would unmap and remap it at every synchronisation).
-    cudaMemPoolProps props;
-    memset(&props, 0, sizeof props);
-    props.allocType = cudaMemAllocationTypePinned;
-    props.location.type = cudaMemLocationTypeDevice;
-    props.location.id = dev;
-    if ((e = cudaMemPoolCreate(&ix->pool, &props)) != cudaSuccess) {
-        rc = report_cuda(e, "psb_build_ex: cudaMemPoolCreate");
-        ix->pool = nullptr;
+    if ((rc = make_pool(ix, "psb_build_ex")) != PSB_OK) {
         index_release(ix);
         return rc;
     }
-    uint64_t keep = UINT64_MAX;
-    cudaMemPoolSetAttribute(ix->pool, cudaMemPoolAttrReleaseThreshold, &keep);
     *out = ix;
     return PSB_OK;
 }
@@ -276,14 +288,14 @@ static void *mapped_host_ptr(void *p)
 // staged through stream-ordered device scratch with copies on the same stream.
 static int knn_impl(const char *fn, const psb_index *ix, const float *queries, int64_t q, int32_t k,
                     int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant,
-                    int64_t *stats, int parts = 1)
+                    int64_t *stats, int parts = 1, TraceOut tr = TraceOut{nullptr, nullptr, 0})
 {
     g_err[0] = 0;
     int rc = check_query_args(fn, ix, queries, q, k, out_ids, out_dists);
     if (rc != PSB_OK) return rc;
     if (variant & ~(uint32_t)(PSB_VAR_NOCACHE | PSB_VAR_NOMAXDIST | PSB_VAR_INPUT_ORDER | PSB_VAR_LEAF_ORDER |
                               PSB_VAR_PREFETCH_NEXT | PSB_VAR_PREFETCH_IDS | PSB_VAR_P1_INDEX_TIE |
-                              PSB_VAR_KTH_MAXDIST | PSB_VAR_NO_AUTO_PREFETCH)) {
+                              PSB_VAR_KTH_MAXDIST | PSB_VAR_NO_AUTO_PREFETCH | PSB_VAR_GENERIC_D)) {
         psb_set_error("%s: unknown variant bits 0x%x", fn, variant);
         return PSB_EINVAL;
     }
@@ -291,7 +303,7 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
         psb_set_error("%s: unknown algo %d", fn, algo);
         return PSB_EINVAL;
     }
-    if (stats && algo == PSB_ALGO_BRUTE) {
+    if ((stats || tr.len) && algo == PSB_ALGO_BRUTE) {
         psb_set_error("%s: stats are defined for the tree traversals only", fn);
         return PSB_EINVAL;
     }
@@ -334,7 +346,7 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
     if (rc == PSB_OK) {
         const DevIndex v = dev_view(ix);
         rc = algo == PSB_ALGO_BRUTE ? psb::launch_brute(v, dq, q, k, di, dd, st, ix->sm_count, ix->pool)
-                                    : psb::launch_tree(algo, v, dq, q, k, di, dd, st, variant, stats, ix->pool, parts);
+                                    : psb::launch_tree(algo, v, dq, q, k, di, dd, st, variant, stats, ix->pool, parts, tr);
     }
     if (staged) {
         if (rc == PSB_OK && ((e = cudaMemcpyAsync(out_ids, di, bo, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||
@@ -362,6 +374,22 @@ int psb_knn_stats(const psb_index *ix, const float *queries, int64_t q, int32_t 
         return PSB_EINVAL;
     }
     return knn_impl("psb_knn_stats", ix, queries, q, k, out_ids, out_dists, stream, algo, variant, stats);
+}
+
+int psb_knn_trace(const psb_index *ix, const float *queries, int64_t q, int32_t k, int32_t *out_ids,
+                  float *out_dists, void *stream, int32_t algo, uint32_t variant, int64_t *stats, int64_t *trace,
+                  int32_t cap, int32_t *trace_len)
+{
+    if (q > 0 && (!trace || !trace_len || cap < 1)) {
+        psb_set_error("psb_knn_trace: trace / trace_len NULL or cap < 1");
+        return PSB_EINVAL;
+    }
+    if (q > 0 && (!is_device_ptr(trace) || !is_device_ptr(trace_len) || (stats && !is_device_ptr(stats)))) {
+        psb_set_error("psb_knn_trace: trace, trace_len and stats must be device memory");
+        return PSB_EINVAL;
+    }
+    return knn_impl("psb_knn_trace", ix, queries, q, k, out_ids, out_dists, stream, algo, variant, stats, 1,
+                    TraceOut{trace, trace_len, cap});
 }
 
 int psb_knn_split(const psb_index *ix, const float *queries, int64_t q, int32_t k, int32_t parts,
@@ -459,6 +487,142 @@ int psb_index_export(const psb_index *ix, void *host_buf, int64_t cap, int64_t *
         (e = cudaMemcpy(p + bp, ix->ids, bi, cudaMemcpyDeviceToHost)) != cudaSuccess ||
         (e = cudaMemcpy(p + bp + bi, ix->nodes, 4 * (size_t)ix->node_floats, cudaMemcpyDeviceToHost)) != cudaSuccess)
         return report_cuda(e, "psb_index_export");
+    return PSB_OK;
+}
+
+// Upload an export blob as an index (replicas: build once, broadcast the blob;
+// tests: hand-built trees). Everything the exactness argument rests on is
+// checked first: the level geometry of a packed tree, finite coordinates for
+// real points and +inf for pad slots (id -1), and every box containing what is
+// below it (App. C of SURVEY.md: then MINDIST <= dist <= MAXDIST holds under
+// RN rounding for every point beneath).
+int psb_index_import(const void *blob, int64_t size, psb_index **out)
+{
+    g_err[0] = 0;
+    if (!out || !blob) { psb_set_error("psb_index_import: NULL argument"); return PSB_EINVAL; }
+    *out = nullptr;
+    if (size < 64) { psb_set_error("psb_index_import: blob too small"); return PSB_EINVAL; }
+    const char *b = (const char *)blob;
+    int64_t hdr[8];
+    memcpy(hdr, b, sizeof hdr);
+    const int64_t n_hdr = hdr[0], L = hdr[3], id_base = hdr[5], total = hdr[6];
+    const int64_t d64 = hdr[1], F64 = hdr[2], H64 = hdr[4];
+    if (hdr[7] != 0) { psb_set_error("psb_index_import: sphere indexes cannot be imported"); return PSB_EUNSUPPORTED; }
+    if (d64 < 1 || d64 > PSB_DMAX || H64 < 1 || H64 > PSB_MAXLVL || L < 1 || L > ((int64_t)1 << 31) / 32) {
+        psb_set_error("psb_index_import: header out of range");
+        return PSB_EINVAL;
+    }
+    const int32_t d = (int32_t)d64, F = (int32_t)F64, H = (int32_t)H64;
+    GpuLayoutShape shape;
+    int rc = psb_layout_shape(L * F64, d, F, 0, 0, &shape);   // validates d and F
+    if (rc != PSB_OK) return rc;
+    if (size < 64 + 8 * (H64 + 1)) { psb_set_error("psb_index_import: blob too small"); return PSB_EINVAL; }
+    int64_t nlev[PSB_MAXLVL + 1] = {};
+    memcpy(nlev, b + 64, 8 * (size_t)(H + 1));
+    if (shape.H != H || shape.L != L || shape.total_node_floats / (2 * d64 * F64) != total) {
+        psb_set_error("psb_index_import: level geometry is not that of a packed tree with %lld leaves", (long long)L);
+        return PSB_EINVAL;
+    }
+    for (int l = 0; l <= H; ++l)
+        if (nlev[l] != shape.nlev[l]) { psb_set_error("psb_index_import: nodes_per_level[%d] wrong", l); return PSB_EINVAL; }
+    if (size != blob_size(L, d, F, H, shape.total_node_floats)) {
+        psb_set_error("psb_index_import: size %lld does not match the header", (long long)size);
+        return PSB_EINVAL;
+    }
+    const float *pts = (const float *)(b + 64 + 8 * (H + 1));
+    const int32_t *ids = (const int32_t *)(pts + L * d64 * F64);
+    const float *nodes = (const float *)(ids + L * F64);
+    // points: real slots finite with an id >= 0, pad slots +inf with id -1
+    int64_t n_real = 0;
+    bool irregular = false;
+    for (int64_t j = 0; j < L; ++j) {
+        int64_t cnt = 0;
+        for (int s = 0; s < F; ++s) {
+            const int32_t id = ids[j * F + s];
+            if (id < -1) { psb_set_error("psb_index_import: id %d < -1", id); return PSB_EINVAL; }
+            for (int c = 0; c < d; ++c) {
+                const float v = pts[(j * d + c) * F + s];
+                if (id >= 0 ? !std::isfinite(v) : !(std::isinf(v) && v > 0)) {
+                    psb_set_error("psb_index_import: leaf %lld slot %d: coordinates must be finite for a point "
+                                  "and +inf for a pad slot", (long long)j, s);
+                    return PSB_EINVAL;
+                }
+            }
+            cnt += id >= 0;
+        }
+        n_real += cnt;
+        if (j + 1 < L && cnt < F) irregular = true;
+    }
+    if (n_real != n_hdr || n_real < 1) {
+        psb_set_error("psb_index_import: header n=%lld but %lld real points", (long long)n_hdr, (long long)n_real);
+        return PSB_EINVAL;
+    }
+    // boxes: child c of node (l, i) is (l-1, i*F + c); its box must contain the
+    // points of leaf i*F + c (l = 1) or the boxes of that node's children (l >= 2)
+    const int64_t blk = 2 * d64 * F64;
+    for (int l = 1; l <= H; ++l) {
+        const float *cur = nodes + shape.level_off[l];
+        for (int64_t i = 0; i < nlev[l]; ++i) {
+            for (int c = 0; c < F; ++c) {
+                const int64_t g = i * F + c;
+                for (int dd = 0; dd < d; ++dd) {
+                    const float lo = cur[i * blk + (2 * dd) * F + c], hi = cur[i * blk + (2 * dd + 1) * F + c];
+                    if (std::isnan(lo) || std::isnan(hi)) { psb_set_error("psb_index_import: NaN box"); return PSB_EINVAL; }
+                    float mn = INFINITY, mx = -INFINITY;
+                    if (g < nlev[l - 1]) {
+                        if (l == 1) {
+                            for (int s = 0; s < F; ++s)
+                                if (ids[g * F + s] >= 0) {
+                                    mn = std::min(mn, pts[(g * d + dd) * F + s]);
+                                    mx = std::max(mx, pts[(g * d + dd) * F + s]);
+                                }
+                        } else {
+                            const float *cb = nodes + shape.level_off[l - 1] + g * blk;
+                            for (int s = 0; s < F; ++s) {
+                                mn = std::min(mn, cb[(2 * dd) * F + s]);
+                                mx = std::max(mx, cb[(2 * dd + 1) * F + s]);
+                            }
+                        }
+                    }
+                    const bool empty = mn > mx;
+                    if (empty ? !(std::isinf(lo) && lo > 0 && std::isinf(hi) && hi < 0) : (lo > mn || hi < mx)) {
+                        psb_set_error("psb_index_import: box of child %d of node %lld at level %d does not bound "
+                                      "its content (dim %d)", c, (long long)i, l, dd);
+                        return PSB_EINVAL;
+                    }
+                }
+            }
+        }
+    }
+    int dev = -1;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return report_cuda(e, "psb_index_import: cudaGetDevice");
+    psb_index *ix = new (std::nothrow) psb_index;
+    if (!ix) { psb_set_error("psb_index_import: host allocation failed"); return PSB_ENOMEM; }
+    ix->device = dev;
+    cudaDeviceGetAttribute(&ix->sm_count, cudaDevAttrMultiProcessorCount, dev);
+    ix->n = n_real; ix->L = L; ix->id_base = id_base;
+    ix->d = d; ix->F = F; ix->H = H;
+    for (int l = 0; l <= PSB_MAXLVL; ++l) { ix->nlev[l] = shape.nlev[l]; ix->level_off[l] = shape.level_off[l]; }
+    ix->node_floats = shape.total_node_floats;
+    ix->blk_floats = (int32_t)blk;
+    ix->irregular = irregular ? 1 : 0;
+    const size_t bp = 4 * (size_t)(L * d64 * F64), bi = 4 * (size_t)(L * F64), bn = 4 * (size_t)shape.total_node_floats;
+    if ((e = cudaMalloc((void **)&ix->pts, bp)) != cudaSuccess || (e = cudaMalloc((void **)&ix->ids, bi)) != cudaSuccess ||
+        (e = cudaMalloc((void **)&ix->nodes, bn)) != cudaSuccess ||
+        (e = cudaMemcpy(ix->pts, pts, bp, cudaMemcpyHostToDevice)) != cudaSuccess ||
+        (e = cudaMemcpy(ix->ids, ids, bi, cudaMemcpyHostToDevice)) != cudaSuccess ||
+        (e = cudaMemcpy(ix->nodes, nodes, bn, cudaMemcpyHostToDevice)) != cudaSuccess) {
+        rc = report_cuda(e, "psb_index_import: upload");
+        index_release(ix);
+        return rc;
+    }
+    ix->device_bytes = (int64_t)(bp + bi + bn);
+    if ((rc = make_pool(ix, "psb_index_import")) != PSB_OK) {
+        index_release(ix);
+        return rc;
+    }
+    *out = ix;
     return PSB_OK;
 }
 

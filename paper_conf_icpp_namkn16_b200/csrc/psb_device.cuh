@@ -279,6 +279,10 @@ __device__ __forceinline__ void sphere_bounds(const float *__restrict__ blk, con
             }
         }
     });
+    if (!MAX) {
+#pragma unroll
+        for (int t = 0; t < V; ++t) Md[t] = 0.f;   // defined for callers that read it (closest_child)
+    }
     float r[V];
     ldv<V>(blk + d * F + lane * V, r);
     const float g = __fmul_ru((float)(2 * d + 4), 5.9604644775390625e-8f);   // (2d+4) 2^-24
@@ -530,18 +534,33 @@ __device__ __forceinline__ int64_t global_ns()
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return (int64_t)t;
 }
+// Traversal trace (psb_knn_trace): one int64 per step of a query's walk, in
+// order: node | level << 32 | flags << 40 (include/psb.h PSB_TRACE_*).
+enum : unsigned { TR_PASS1 = 1u, TR_CHANGED = 2u, TR_SKIPPED = 4u, TR_FETCHED = 8u };
 template <bool ON>
 struct Stats {
     uint32_t fetch = 0, hit = 0, leaf = 0, ids = 0, offers = 0, cand = 0;
     int64_t t0 = 0;   // %globaltimer at the query's start (in-batch service time)
+    int32_t nstep = 0;
     __device__ __forceinline__ Stats() { if (ON) t0 = global_ns(); }
     __device__ __forceinline__ void node(bool fetched) { if (ON) { fetched ? ++fetch : ++hit; } }
     __device__ __forceinline__ void scan() { if (ON) ++leaf; }
     __device__ __forceinline__ void id_loads(int n) { if (ON) ids += n; }
     __device__ __forceinline__ void merged(int m) { if (ON) { cand += m; offers += m > 0; } }
-    __device__ __forceinline__ void write(int64_t *st, int64_t qi, int lane) const
+    // one traversal step: internal node (lvl >= 1) or leaf (lvl = 0)
+    __device__ __forceinline__ void step(const TraceOut &tr, int64_t qi, int lane, int lvl, int node, unsigned flags)
+    {
+        if (ON) {
+            if (tr.buf && lane == 0 && nstep < tr.cap)
+                tr.buf[qi * tr.cap + nstep] = (int64_t)(uint32_t)node | ((int64_t)lvl << 32) | ((int64_t)flags << 40);
+            ++nstep;
+        }
+    }
+    __device__ __forceinline__ void write(int64_t *st, const TraceOut &tr, int64_t qi, int lane) const
     {
         if (ON && lane == 0) {
+            if (tr.len) tr.len[qi] = nstep;
+            if (!st) return;
             int64_t *o = st + qi * 8;
             o[0] = fetch;   // internal-node blocks fetched from memory
             o[1] = leaf;    // leaf blocks scanned
@@ -646,8 +665,11 @@ __device__ __forceinline__ bool scan_leaf(const DevIndex &ix, int leaf, const Qu
     // next leaf whenever this scan changes the list (Alg. 1 l.41), and this leaf's
     // ids are needed as soon as a distance passes the filter: start both L2->L1
     // transfers now, without holding registers.
-    if ((pf & PF_NEXT) && leaf + 1 < ix.L && lane < ix.d * V)
-        asm volatile("prefetch.global.L1 [%0];" ::"l"(ix.pts + ((int64_t)leaf + 1) * ix.d * F + lane * 32));
+    if ((pf & PF_NEXT) && leaf + 1 < ix.L) {
+        // the whole right-sibling block: d*V lines of 128 B
+        for (int o = lane; o < ix.d * V; o += 32)
+            asm volatile("prefetch.global.L1 [%0];" ::"l"(ix.pts + ((int64_t)leaf + 1) * ix.d * F + o * 32));
+    }
     if ((pf & PF_IDS) && lane < V)
         asm volatile("prefetch.global.L1 [%0];" ::"l"(ix.ids + (int64_t)leaf * F + lane * 32));
     constexpr int DC = D;   // compile-time d (0: runtime)

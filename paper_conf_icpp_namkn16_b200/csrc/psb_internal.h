@@ -30,9 +30,19 @@ struct DevIndex {
     int32_t sm_count;                   // of the index's device (launch sizing)
     int32_t sphere;                     // 0: MBR node blocks [d][2][F]; 1: sphere blocks [d+1][F]
     int32_t blk_floats;                 // floats per internal node block
+    int32_t irregular;                  // imported tree whose leaves are not all full (but the last):
+                                        // the count-aware MAXDIST bound (R3) does not apply
     // per launch (k known): a child (lvl-1, c) of a level-lvl node holds >= k points
     // iff c <= kcnt_lim[lvl] (every subtree but the level's last holds >= F points)
     int32_t kcnt_lim[PSB_MAXLVL + 1];
+};
+
+// psb_knn_trace output: per query, its traversal steps in order (kernels with
+// counting compiled in only). buf [q][cap] (nullable), len [q] (nullable).
+struct TraceOut {
+    int64_t *buf;
+    int32_t *len;
+    int cap;
 };
 
 // Level geometry of a packed tree (shared by the host and GPU loaders).

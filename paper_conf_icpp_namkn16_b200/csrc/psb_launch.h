@@ -13,8 +13,11 @@ int report_cuda(cudaError_t e, const char *what);
 // `stats` (nullable, device [nq][4] int64): per query {internal node fetches,
 // leaf scans, id loads, path-cache hits}.
 // parts > 1 (PSB only): latency mode, each query's leaves split over `parts` warps.
+// `tr` (psb_knn_trace): per-query traversal steps; with stats or tr.len set the
+// counting instantiation runs (PSB_VAR_GENERIC_D: the generic-d one).
 int launch_tree(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool, int parts);
+                float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool, int parts,
+                const TraceOut &tr);
 
 // Exhaustive scan of all points (knn_brute.cu). Splits the point set into
 // chunks when there are too few queries to fill the GPU and merges the partial
@@ -28,7 +31,8 @@ int launch_brute(const DevIndex &ix, const float *queries, int64_t nq, int k, in
 constexpr int PSB_NOT_INSTANTIATED = 1;
 template <int D, int V>
 int launch_tree_ks(int algo, const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi,
-                   float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool, int parts);
+                   float *od, cudaStream_t st, uint32_t variant, int64_t *stats, cudaMemPool_t pool, int parts,
+                   const TraceOut &tr);
 template <int D, int V>
 int launch_brute_ks(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi, float *od,
                     cudaStream_t st, int sm, cudaMemPool_t pool);

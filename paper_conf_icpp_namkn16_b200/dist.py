@@ -48,21 +48,28 @@ def allgather_topk(ids: torch.Tensor, dists: torch.Tensor, group=None):
 
 def data_sharded_knn(local_knn: Callable, merge: Callable, queries: torch.Tensor, k: int,
                      group=None, merge_all: bool = False):
-    """One data-sharded step: local kNN over this rank's slab (ids already
-    global via id_base), all-gather of the [q, k] lists, exact merge.
+    """One data-sharded step (the NCCL route): local kNN over this rank's slab(s)
+    (ids already global via id_base), all-gather of the lists, exact merge.
 
+    `local_knn(queries, k)` returns this rank's lists as [q, k] (one slab) or
+    [s, q, k] (s slabs held by this rank); the all-gather stacks every rank's
+    lists into [world*s, q, k] and `merge` (psb_merge_topk) combines them.
     Returns (ids, dists) for this rank's query slice (or for all queries when
     merge_all). Exact because (dist, id) is a total order and every global id
     lives in exactly one slab."""
     world = dist.get_world_size(group)
     rank = dist.get_rank(group)
     ids, dists = local_knn(queries, k)
-    if world == 1:
-        return ids, dists
-    gi, gd = allgather_topk(ids, dists, group)
+    if ids.dim() == 2:
+        if world == 1:
+            return ids, dists
+        ids, dists = ids.unsqueeze(0), dists.unsqueeze(0)
+    s, q = ids.shape[0], ids.shape[1]
+    gi, gd = allgather_topk(ids, dists, group)                 # [world, s, q, k]
+    gi, gd = gi.reshape(world * s, q, k), gd.reshape(world * s, q, k)
     if merge_all:
         return merge(gi, gd, k)
-    sl = query_slice(queries.shape[0], world, rank)
+    sl = query_slice(q, world, rank)
     return merge(gi[:, sl].contiguous(), gd[:, sl].contiguous(), k)
 
 
@@ -102,14 +109,61 @@ def peer_exchange(q: int, k: int, group=None):
     return ex
 
 
-def data_sharded_knn_p2p(ex, index, queries: torch.Tensor, algo: int = 0, variant: int = 0, stream=None):
+def chunk_rows(q: int, parts: int, rank: int, chunks: int) -> list[slice]:
+    """Rows a rank merges in chunked data-sharded mode: its 1/parts slice of each
+    of `chunks` contiguous chunks of the batch, in chunk order (chunks = 1: the
+    plain query_slice)."""
+    cb = shard_bounds(q, max(1, chunks))
+    out = []
+    for c in range(max(1, chunks)):
+        sl = query_slice(cb[c + 1] - cb[c], parts, rank)
+        out.append(slice(cb[c] + sl.start, cb[c] + sl.stop))
+    return out
+
+
+_side_streams: dict = {}
+
+
+def _side_stream():
+    dev = torch.cuda.current_device()
+    if dev not in _side_streams:
+        _side_streams[dev] = torch.cuda.Stream()
+    return _side_streams[dev]
+
+
+def data_sharded_knn_p2p(ex, index, queries: torch.Tensor, algo: int = 0, variant: int = 0, stream=None,
+                         chunks: int = 1, side=None, out=None):
     """One data-sharded step without a collective: local search into this rank's
-    exchange buffers, then one kernel that waits for every peer's flag and merges
-    this rank's query slice straight out of all ranks' buffers over NVLink.
-    Returns (ids, dists) for the slice query_slice(q, world, rank)."""
-    ex.local_knn(index, queries, algo=algo, variant=variant, stream=stream)
-    sl = query_slice(ex.q, ex.parts, ex.rank)
-    return ex.step(sl.start, sl.stop - sl.start, stream=stream)
+    exchange buffers, then kernels that wait for every peer's flag and merge this
+    rank's rows straight out of all ranks' buffers over NVLink.
+
+    chunks = 1: search all q queries, then merge query_slice(q, world, rank).
+    chunks > 1: the batch is cut into `chunks` pieces; chunk c is searched and
+    signalled on `stream` while the merge of chunk c-1 runs on a second stream
+    (`side`), so the exchange overlaps the search; this rank merges its slice of
+    every chunk (chunk_rows). Returns (ids, dists) of those rows, in order."""
+    main = stream if stream is not None else torch.cuda.current_stream()
+    rows = chunk_rows(ex.q, ex.parts, ex.rank, chunks)
+    total = sum(r.stop - r.start for r in rows)
+    if out is None:
+        out = (torch.empty((total, ex.k), dtype=torch.int32, device=queries.device),
+               torch.empty((total, ex.k), dtype=torch.float32, device=queries.device))
+    if chunks <= 1:
+        ex.local_knn(index, queries, algo=algo, variant=variant, stream=main)
+        return ex.step(rows[0].start, total, stream=main, out=out)
+    side = side if side is not None else _side_stream()
+    ex.begin()
+    side.wait_stream(main)                     # out buffers / previous epoch in stream order
+    cb = shard_bounds(ex.q, chunks)
+    o = 0
+    for c in range(chunks):
+        ex.local_knn(index, queries, algo=algo, variant=variant, stream=main, rows=slice(cb[c], cb[c + 1]))
+        ex.signal(cb[c + 1], stream=main)
+        n = rows[c].stop - rows[c].start
+        ex.merge(rows[c].start, n, stream=side, out=(out[0][o:o + n], out[1][o:o + n]))
+        o += n
+    main.wait_stream(side)                     # results (and the next epoch) after every merge
+    return out
 
 
 def build_shard(points, fanout: int, world: int, rank: int, packing: int = 0):

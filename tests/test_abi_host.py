@@ -18,7 +18,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 def test_exports_every_declared_symbol():
     hdr = open(os.path.join(ROOT, "include", "psb.h")).read()
-    declared = set(re.findall(r"\b(psb_[a-z_]+)\s*\(", hdr))
+    declared = set(re.findall(r"\b(psb_[a-z0-9_]+)\s*\(", hdr))
     assert declared == set(psb.EXPORTS)
     assert all(psb.symbols_exported().values())
     assert "sm_100a" in psb.psb_version()

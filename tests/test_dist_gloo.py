@@ -62,6 +62,23 @@ def _worker(rank, world, port, mode, out):
         ids2, d2 = pd.data_sharded_knn(local, _np_merge, qs, k, merge_all=True)
         exp2 = oracle.knn_bruteforce(pts, qs.numpy(), k)
         ok = ok and np.array_equal(ids2.numpy(), exp2[0])
+    elif mode == "data_multi":
+        # each rank holds two slabs: local returns [2, q, k], the all-gather stacks [world*2, q, k]
+        b = pd.shard_bounds(len(pts), 2 * world)
+
+        def local(q, kk):
+            outs_i, outs_d = [], []
+            for s in (2 * rank, 2 * rank + 1):
+                ids, d = oracle.knn_bruteforce(pts[b[s]:b[s + 1]], q.numpy(), kk)
+                outs_i.append(np.where(ids >= 0, ids + b[s], -1).astype(np.int32))
+                outs_d.append(d)
+            return torch.from_numpy(np.stack(outs_i)), torch.from_numpy(np.stack(outs_d))
+
+        ids, d = pd.data_sharded_knn(local, _np_merge, qs, k)
+        sl = pd.query_slice(len(qs), world, rank)
+        exp = oracle.knn_bruteforce(pts, qs.numpy()[sl], k)
+        ok = np.array_equal(ids.numpy(), exp[0]) and np.array_equal(d.numpy().view(np.uint32),
+                                                                     exp[1].view(np.uint32))
     else:
         def local(q, kk):
             ids, d = oracle.knn_bruteforce(pts, q.numpy(), kk)
@@ -75,7 +92,7 @@ def _worker(rank, world, port, mode, out):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("mode", ["data", "query"])
+@pytest.mark.parametrize("mode", ["data", "data_multi", "query"])
 def test_two_rank_modes(mode):
     mgr = mp.Manager()
     out = mgr.dict()
@@ -91,3 +108,22 @@ def test_shard_bounds_cover_exactly():
             assert b[0] == 0 and b[-1] == n and all(b[i] <= b[i + 1] for i in range(w))
             sizes = [b[i + 1] - b[i] for i in range(w)]
             assert max(sizes) - min(sizes) <= 1
+
+
+def test_chunk_rows_partition_the_batch():
+    """Chunked data-sharded mode: the rows the ranks merge cover every query
+    exactly once, each rank's rows come chunk by chunk, and chunks = 1 is the
+    plain query_slice."""
+    from paper_conf_icpp_namkn16_b200 import dist as pd
+    for q in (1, 3, 1000, 1_000_000):
+        for P in (1, 2, 3, 8):
+            for C in (1, 2, 5, 16):
+                cover = np.zeros(q, np.int32)
+                for r in range(P):
+                    rows = pd.chunk_rows(q, P, r, C)
+                    assert len(rows) == C
+                    for s in rows:
+                        cover[s] += 1
+                    if C == 1:
+                        assert rows[0] == pd.query_slice(q, P, r)
+                assert (cover == 1).all()
