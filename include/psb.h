@@ -176,10 +176,10 @@ int psb_knn_bruteforce(const psb_index *idx, const float *queries, int64_t q, in
  *                          smallest MAXDIST over children whose subtrees hold
  *                          >= k points (R3): tighter, and a warp min
  *                          instead of a radix select.
- * bit 8 PSB_VAR_NO_AUTO_PREFETCH — PSB at compile-time d = 16 turns both
- *                          prefetches (bits 4 and 5) on by default (measured
- *                          faster there, slower at d <= 8); this
- *                          bit keeps them off unless bits 4/5 ask for them.
+ * bit 8 PSB_VAR_NO_AUTO_PREFETCH — a build with PSB_AUTO_PREFETCH_MIN_D set
+ *                          turns bits 4 and 5 on for compile-time d >= that
+ *                          value; this bit keeps them off. The default build
+ *                          sets no such d (measured slower).
  * bit 9 PSB_VAR_GENERIC_D — run the runtime-d instantiation of the kernels even
  *                          where a compile-time-d one exists (d, fanout) in
  *                          {(2,32), (3,64), (3,128), (8,128), (16,128)}: the two

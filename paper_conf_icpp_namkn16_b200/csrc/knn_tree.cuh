@@ -27,14 +27,15 @@ constexpr double REORDER_MIN_BYTES = 64.0 * (1 << 20);
 #ifndef PSB_MINBLOCKS_LARGE_D
 #define PSB_MINBLOCKS_LARGE_D 6
 #endif
-// PSB prefetches the right sibling's coordinates and the scanned leaf's ids by
-// default at compile-time d >= this (PSB_VAR_NO_AUTO_PREFETCH turns it off): the
-// 8 KB leaf blocks of d = 16 make the long queries that end a C4 batch
-// load-latency bound (C4 16.9 -> 15.9 ms), while at d <= 8 the traversal is
-// issue bound and a prefetch is a wasted L1 fill (C3 6.59 -> 7.08 ms with it;
-// profiles/r01_prefetch.md).
+// PSB prefetched the right sibling's coordinates and the scanned leaf's ids by
+// default at compile-time d >= this in round 1 (C4 16.9 -> 15.9 ms, when the
+// prefetch covered only half of the 8 KB leaf block). Covering the whole block
+// (every line of it) made it a loss: C4 15.3-15.5 ms without it, 16.5-16.7 with
+// both prefetches, 15.6 with the ids alone, 16.3-16.4 with the next leaf alone
+// (profiles/r02_experiments.md). So no d turns it on by default; the variant
+// bits PSB_VAR_PREFETCH_NEXT / _IDS still do.
 #ifndef PSB_AUTO_PREFETCH_MIN_D
-#define PSB_AUTO_PREFETCH_MIN_D 16
+#define PSB_AUTO_PREFETCH_MIN_D 1024   // off: no compile-time d turns the prefetch on
 #endif
 template <int D>
 struct MinBlocks {
