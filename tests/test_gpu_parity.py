@@ -146,29 +146,59 @@ def test_query_order_generic_d_and_sphere():
         idx.free()
 
 
-def test_c3_sampled():
-    """configs[2]: 8-D uniform n=4M F=128 k=16; a 2,000-query sample of the 10^5."""
+def test_c3_full_batch_sampled():
+    """configs[2]: 8-D uniform n=4M F=128 k=16, the bench's default workload, in the
+    launch configuration bench.py times (all 10^5 queries in one launch: closest-leaf
+    order, persistent grid); 2,000 rows spread over the batch against the oracle's
+    B&B, 40 against its brute force."""
     cfg = W.config("C3")
     pts = cfg.points()
-    qs = cfg.queries(q=2000)
+    qs = cfg.queries()
     idx = _psb().psb_build(pts, cfg.fanout)
-    exp = oracle.Tree(pts).knn(qs, cfg.k)
-    for algo in ALGOS:
-        assert_same(run(idx, qs, cfg.k, algo), exp, f"C3 {algo}")
-    bf = oracle.knn_bruteforce(pts, qs[:40], cfg.k)
-    assert_same(run(idx, qs[:40], cfg.k), bf, "C3 psb vs oracle brute")
+    sub = np.arange(0, len(qs), len(qs) // 2000)
+    exp = oracle.Tree(pts).knn(qs[sub], cfg.k)
+    for algo in ("psb", "bnb"):
+        gi, gd = run(idx, qs, cfg.k, algo)
+        assert_same((gi[sub], gd[sub]), exp, f"C3 {algo} (full batch)")
+    gi, gd = run(idx, qs[:2000], cfg.k, "brute")
+    assert_same((gi[sub[sub < 2000]], gd[sub[sub < 2000]]), (exp[0][: (sub < 2000).sum()], exp[1][: (sub < 2000).sum()]),
+                "C3 brute")
+    bf = oracle.knn_bruteforce(pts, qs[sub[:40]], cfg.k)
+    gi, gd = run(idx, qs, cfg.k)
+    assert_same((gi[sub[:40]], gd[sub[:40]]), bf, "C3 psb vs oracle brute")
     idx.free()
 
 
-def test_c4_sampled():
-    """configs[3]: 16-D clustered n=16M F=128 k=64; 200 sampled queries."""
+def test_c4_full_batch_all_rows():
+    """configs[3]: 16-D clustered n=16M F=128 k=64, in the launch configuration
+    bench.py times: all 10^4 queries in one launch, in closest-leaf order; every row
+    against the oracle's B&B (PSB and B&B; brute force on 200 queries)."""
     cfg = W.config("C4")
     pts = cfg.points()
-    qs = cfg.queries(q=200)
+    qs = cfg.queries()
     idx = _psb().psb_build(pts, cfg.fanout)
     exp = oracle.Tree(pts).knn(qs, cfg.k)
-    for algo in ALGOS:
-        assert_same(run(idx, qs, cfg.k, algo), exp, f"C4 {algo}")
+    for algo in ("psb", "bnb"):
+        assert_same(run(idx, qs, cfg.k, algo), exp, f"C4 {algo} (full batch)")
+    assert_same(run(idx, qs[:200], cfg.k, "brute"), (exp[0][:200], exp[1][:200]), "C4 brute")
+    idx.free()
+
+
+def test_c5_slab_full_batch_sampled():
+    """configs[4], one GPU's share of the data-sharded C5: slab 0 of 8 (64M 3-D
+    uniform points, ids 0..64M-1), F=128, k=32, in the launch configuration bench.py
+    times (all 10^6 queries in one launch); 2,000 rows spread over the batch against
+    the oracle's B&B over the same slab."""
+    cfg = W.config("C5")
+    n = cfg.n // 8
+    pts = cfg.points(n=n, row0=0)
+    qs = cfg.queries()
+    idx = _psb().psb_build_ex(pts, cfg.fanout, id_base=0)
+    sub = np.arange(0, len(qs), len(qs) // 2000)
+    exp = oracle.Tree(pts).knn(qs[sub], cfg.k)
+    for algo in ("psb", "bnb"):
+        gi, gd = run(idx, qs, cfg.k, algo)
+        assert_same((gi[sub], gd[sub]), exp, f"C5 slab {algo} (full batch)")
     idx.free()
 
 
