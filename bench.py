@@ -150,9 +150,10 @@ def issue_peak() -> float:
 
 
 def alu_peak() -> float:
-    """FP32 lane-instruction ceiling, T lane-inst/s: 148 SMs x 4 SMSPs x 32 lanes x
-    1 warp instruction per cycle at the max SM clock (B200_PROFILING.md,
-    MEASURED_PEAKS.json sm_max_mhz); DESIGN.md §6 derives it."""
+    """FP32 arithmetic ceiling, T ops/s (an add, a subtract or a multiply each one
+    op): 148 SMs x 128 FP32 lanes x the max SM clock (MEASURED_PEAKS.json
+    sm_max_mhz) = 148 x 4 SMSPs x one packed pair instruction (64 ops) per 2
+    cycles; DESIGN.md §6 derives it."""
     return issue_peak() * 32 / 1e3
 
 
@@ -265,11 +266,13 @@ def roofline(algo, idx, q, k, alg_bytes, kern_s, prof_cfg, l2_peak):
     (packed subtract / square / add pairs) against the lane-instruction ceiling."""
     hbm, hbm_src = peaks()
     if algo == "brute":
-        ops = 1.5 * idx.n * q * idx.d
+        ops = 3.0 * idx.n * q * idx.d
         a = ops / kern_s / 1e12
-        prim = {"bound": "alu", "achieved": a, "peak": alu_peak(), "unit": "T lane-inst/s", "frac": a / alu_peak(),
-                "algorithmic_lane_inst_per_launch": ops,
-                "peak_source": "148 SMs x 4 SMSPs x 32 lanes x 1 inst/cycle x sm_max_mhz (DESIGN.md §6)"}
+        prim = {"bound": "alu", "achieved": a, "peak": alu_peak(), "unit": "T FP32-op/s", "frac": a / alu_peak(),
+                "algorithmic_fp32_ops_per_launch": ops,
+                "peak_source": "148 SMs x 128 FP32 lanes x sm_max_mhz: packed FADD2/FFMA2 pairs issue at one "
+                               "per 2 cycles per SMSP (ncu: fma pipe busy 2 cycles per packed instruction; "
+                               "DESIGN.md §6)"}
     else:
         a = alg_bytes / kern_s / 1e9
         prim = {"bound": "l2", "achieved": a, "peak": l2_peak, "unit": "GB/s", "frac": a / l2_peak,
