@@ -508,7 +508,8 @@ def main():
                                               "(PAPER.md L835-838 'query response time')"}
         # comparators on the same batch (same timing protocol, fewer steps)
         comp = {}
-        for name, a in (("psb", psb.PSB_ALGO_PSB), ("bnb", psb.PSB_ALGO_BNB), ("brute", psb.PSB_ALGO_BRUTE)):
+        for name, a in (("psb", psb.PSB_ALGO_PSB), ("psb_split", -1), ("bnb", psb.PSB_ALGO_BNB),
+                        ("brute", psb.PSB_ALGO_BRUTE)):
             if name == "brute" and idx.n * ql > 2e11:
                 comp[name] = {"skipped": f"n*q = {idx.n * ql:.2e} pairs (minutes per batch)"}
                 continue
@@ -519,7 +520,10 @@ def main():
                 flush.fill_(i & 0xFF)
                 s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 s.record(stream)
-                psb.psb_knn_ex(idx, qd, k, algo=a, out=(out_i, out_d))
+                if a < 0:                              # psb_knn_split, auto parts (tail splitting)
+                    psb.psb_knn_split(idx, qd, k, parts=0, out=(out_i, out_d))
+                else:
+                    psb.psb_knn_ex(idx, qd, k, algo=a, out=(out_i, out_d))
                 e.record(stream)
                 torch.cuda.synchronize()
                 if i >= 2:

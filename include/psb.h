@@ -119,13 +119,19 @@ int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int6
 int psb_knn(const psb_index *idx, const float *queries, int64_t q, int32_t k,
             int32_t *out_ids, float *out_dists, void *stream);
 
-/* Latency mode of psb_knn (SURVEY.md §8(e) "intra-GPU split"): each query's
- * leaves are cut into `parts` contiguous ranges, one warp runs PSB on each range,
- * the warps of a query share their pruning distance through atomicMin, and the
- * per-range lists are merged on the device. Same results as psb_knn; for small
- * batches where one warp per query leaves the GPU idle (single-query latency).
- * parts = 0 picks ~16 warps per SM in total (at least 16 leaves per range);
- * parts = 1 is psb_knn. */
+/* Split mode of psb_knn (SURVEY.md §8(e) "intra-GPU split"): `parts` warps share
+ * each query, each running PSB (Alg. 1) over the leaves it owns; the warps of a
+ * query share their pruning distance through atomicMin and their per-part
+ * lists are merged on the device. Same results as psb_knn.
+ *  - When the (query, part) tasks do not fill the GPU (single queries: latency),
+ *    part p owns the p-th of `parts` contiguous leaf ranges.
+ *  - When they do (batches), part p owns the level-1 nodes n with n % parts == p,
+ *    so the eligible leaves of a query, which cluster in neighbouring nodes, are
+ *    spread over all parts: this shortens the long queries that end a batch.
+ * parts = 0 picks: ~16 warps per SM in total (at least 16 leaves per part) for
+ * q <= 8 x SMs; 2-8 parts for batches of fewer than 128 x SMs queries whose
+ * estimated leaves per query, (1 + (min(k,F)/F)^(1/d))^d, reach 64; else 1.
+ * parts = 1 is psb_knn. For k > 128 psb_knn_split runs as psb_knn. */
 int psb_knn_split(const psb_index *idx, const float *queries, int64_t q, int32_t k, int32_t parts,
                   int32_t *out_ids, float *out_dists, void *stream);
 

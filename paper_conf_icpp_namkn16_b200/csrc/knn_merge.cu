@@ -108,9 +108,49 @@ void init_shared_pd(float *gpd, int64_t nq, cudaStream_t st)
     fill_inf<<<(unsigned)((nq + 255) / 256), 256, 0, st>>>(gpd, nq);
 }
 
+// Few parts per query (split batches): one warp per query over its [parts][k]
+// lists, same filter.
+template <int KS>
+__global__ void __launch_bounds__(128)
+merge_parts_small_kernel(const int32_t *__restrict__ ids, const float *__restrict__ dists,
+                         const float *__restrict__ gpd, int parts, int64_t nq, int k, int32_t *__restrict__ out_ids,
+                         float *__restrict__ out_dists)
+{
+    __shared__ u64 scratch_all[4][32];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t qi = (int64_t)blockIdx.x * 4 + w;
+    if (qi >= nq) return;
+    const float lim = __ldg(gpd + qi);
+    TopK<KS> T;
+    T.init();
+    u64 thr = PAD_KEY;
+    for (int p = 0; p < parts; ++p) {
+        const int64_t row = (qi * parts + p) * (int64_t)k;
+        u64 cand[KS];
+        bool any = false;
+#pragma unroll
+        for (int s = 0; s < KS; ++s) {
+            const int r = s * 32 + lane;
+            const float dv = r < k ? __ldg(dists + row + r) : INFINITY;
+            const bool ok = r < k && dv <= lim;
+            cand[s] = ok ? make_key(dv, __ldg(ids + row + r)) : ~0ull;
+            any |= ok;
+        }
+        if (__any_sync(FULL, any)) T.template offer<KS>(cand, k, lane, thr, scratch_all[w]);
+    }
+    T.store(k, lane, out_ids + qi * k, out_dists + qi * k);
+}
+
 int launch_merge_parts(const int32_t *ids, const float *dists, const float *gpd, int parts, int64_t nq, int k,
                        int32_t *oi, float *od, cudaStream_t st)
 {
+    if (parts <= 8) {
+        const unsigned blocks = (unsigned)((nq + 3) / 4);
+        if (k <= 32) merge_parts_small_kernel<1><<<blocks, 128, 0, st>>>(ids, dists, gpd, parts, nq, k, oi, od);
+        else if (k <= 64) merge_parts_small_kernel<2><<<blocks, 128, 0, st>>>(ids, dists, gpd, parts, nq, k, oi, od);
+        else merge_parts_small_kernel<4><<<blocks, 128, 0, st>>>(ids, dists, gpd, parts, nq, k, oi, od);
+        return report_cuda(cudaGetLastError(), "merge_parts kernel launch");
+    }
     if (k <= 32) merge_parts_kernel<1><<<(unsigned)nq, MP_WARPS * 32, 0, st>>>(ids, dists, gpd, parts, k, oi, od);
     else if (k <= 64) merge_parts_kernel<2><<<(unsigned)nq, MP_WARPS * 32, 0, st>>>(ids, dists, gpd, parts, k, oi, od);
     else merge_parts_kernel<4><<<(unsigned)nq, MP_WARPS * 32, 0, st>>>(ids, dists, gpd, parts, k, oi, od);

@@ -6,6 +6,8 @@
 // Step names S1..S11 follow SURVEY.md §8(a); readings R1..R16 follow DESIGN.md §2.
 #include <cuda_runtime.h>
 
+#include <cstdlib>
+
 #include "psb_device.cuh"
 #include "psb_launch.h"
 
@@ -445,25 +447,36 @@ PSB_TREE_KERNEL(bnb_kernel, bnb_query, false)
 
 
 // ---------------------------------------------------------------------------
-// Latency mode (SURVEY.md §8(e) "intra-GPU split"): the leaves of the tree are
-// cut into `parts` contiguous ranges and one warp runs PSB (or B&B) restricted
-// to each range: children whose leaf range misses [lo, hi) are never eligible,
-// `visited` starts at lo-1 and the walk ends when it passes hi-1. The warps of
-// one query share a pruning distance gpd[qi] through atomicMin on its bits
-// (valid: every warp's k-th distance and k-th-MAXDIST bound is an upper bound on
-// the query's true k-th distance, and distances are >= +0 so their bit
-// patterns order like the values). Each warp writes its own sorted list; the
-// lists are merged afterwards (merge_parts_kernel), keeping only keys with
-// dist <= the final gpd. Exact: a point of the true kNN has dist <= d_k <= gpd
-// at all times, so its leaf is never pruned and its warp keeps it.
+// Split mode (SURVEY.md §8(e) "intra-GPU split"; psb_knn_split, and psb_knn for
+// batches too small to fill the GPU): `parts` warps share one query. Part p
+// owns the level-1 nodes n with n % parts == p and runs PSB (Alg. 1 with the
+// readings of DESIGN.md §2) over their leaves only: at level 2 a child is
+// eligible only if it is owned, and a changed leaf's right sibling is scanned
+// only inside the same level-1 node (else the parent link). Interleaving the
+// nodes, rather than cutting the leaves into contiguous ranges, spreads the
+// eligible leaves of a query (which cluster in a few neighbouring nodes) over
+// all parts. The parts share the query's pruning distance gpd[qi] through
+// atomicMin on its bits (valid: every part's k-th distance and k-th-MAXDIST
+// bound is an upper bound on the query's true k-th distance, and distances are
+// >= +0 so their bit patterns order like the values). Each part writes its own
+// sorted list; the lists are merged afterwards (merge_parts_kernel), keeping only
+// keys with dist <= the final gpd. Exact: a point of the true kNN has dist <= d_k
+// <= gpd at all times; its leaf belongs to one part, whose walk is never pruned
+// away from it, so that part keeps it.
 __device__ __forceinline__ float shared_pd(const float *g) { return __ldcg(g); }
 __device__ __forceinline__ void publish_pd(float *g, float v)
 {
     atomicMin(reinterpret_cast<int *>(g), __float_as_int(v));
 }
 
+// Latency mode (few queries): the leaves are cut into `parts` contiguous ranges
+// and one warp runs PSB restricted to each range: children whose leaf range
+// misses [lo, hi) are never eligible, `visited` starts at lo-1 and the walk ends
+// when it passes hi-1. Same shared pruning distance and merge as below. With
+// thousands of parts per query, short contiguous ranges balance better than
+// whole interleaved nodes (C4 single query 0.25 vs 0.49 ms).
 template <int D, int V, int KS, bool ST, bool SPH>
-__device__ __forceinline__ void psb_part_query(const DevIndex &ix, const float *__restrict__ queries, int64_t qi,
+__device__ __forceinline__ void psb_range_query(const DevIndex &ix, const float *__restrict__ queries, int64_t qi,
                                                int part, int parts, int k, int32_t *__restrict__ part_ids,
                                                float *__restrict__ part_dists, float *__restrict__ gpd,
                                                const WarpState &ws, bool use_cache, bool use_max, int lane)
@@ -569,22 +582,186 @@ __device__ __forceinline__ void psb_part_query(const DevIndex &ix, const float *
     T.store(k, lane, oi, od);
 }
 
+// Batch mode (psb_knn_split with many queries): part p owns the level-1 nodes n
+// with n % parts == p (see the comment above shared_pd).
 template <int D, int V, int KS, bool ST, bool SPH>
+__device__ __forceinline__ void psb_node_query(const DevIndex &ix, const float *__restrict__ queries, int64_t qi,
+                                               int part, int parts, int k, int32_t *__restrict__ part_ids,
+                                               float *__restrict__ part_dists, float *__restrict__ gpd,
+                                               const WarpState &ws, bool use_cache, bool use_max, int lane)
+{
+    constexpr int F = 32 * V;
+    constexpr int LOGF = Log2<F>::value;
+    const int H = ix.H;
+    const int L = (int)ix.L;
+    TopK<KS> T;
+    T.init(ws.list, k);
+    int32_t *oi = part_ids + (qi * parts + part) * (int64_t)k;
+    float *od = part_dists + (qi * parts + part) * (int64_t)k;
+    if (H == 1 && part != 0) {                                   // one level-1 node: part 0 owns all
+        T.store(k, lane, oi, od);
+        return;
+    }
+    float *g = gpd + qi;
+    Query<D> q;
+    q.load(queries + qi * ix.d, ix.d, ws.qsmem);
+    for (int l = lane; l <= H; l += 32) ws.cache_node[l] = -1;
+    __syncwarp();
+    u64 thr = PAD_KEY;
+    float pd = shared_pd(g);
+    float published = pd;
+    Stats<ST> S;
+    float *const p1md = ws.cache_md;                             // N*'s child MINDISTs (pass 1)
+    bool pass1 = true;
+    int lvl = H, node = 0, visited = -1;
+    while (true) {
+        if (lvl > 0) {
+            float md[V], Md[V];
+            const float gp = shared_pd(g);                       // issued early, used below
+            internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md, Md);
+            pd = fminf(pd, gp);
+            const int base = node * F;
+            const int c_end = min(F, (int)ix.nlev[lvl - 1] - base);
+            // this lane's children lane*V+t that exist and, at level 2, are owned
+            unsigned mine = 0;
+#pragma unroll
+            for (int t = 0; t < V; ++t) {
+                const int c = lane * V + t;
+                mine |= (unsigned)(c < c_end && (lvl != 2 || (base + c) % parts == part)) << t;
+            }
+            int c = F;
+            if (pass1) {                                         // closest owned child (R4)
+                u64 best = ~0ull;
+#pragma unroll
+                for (int t = 0; t < V; ++t) {
+                    const u64 kk = ((u64)__float_as_uint(md[t]) << 32) | __float_as_uint(Md[t]);
+                    if (((mine >> t) & 1u) && kk < best) best = kk;
+                }
+                best = warp_min_u64(best);
+                // stop descending once the closest owned child lies beyond the shared bound
+                if (best != ~0ull && __uint_as_float((uint32_t)(best >> 32)) <= pd) {
+                    unsigned hit = 0;
+#pragma unroll
+                    for (int t = 0; t < V; ++t) {
+                        const u64 kk = ((u64)__float_as_uint(md[t]) << 32) | __float_as_uint(Md[t]);
+                        hit |= (unsigned)(((mine >> t) & 1u) && kk == best) << t;
+                    }
+                    const unsigned bal = __ballot_sync(FULL, hit != 0);
+                    const int src = __ffs(bal) - 1;
+                    c = src * V + (__ffs(__shfl_sync(FULL, hit, src)) - 1);
+                } else {
+                    pass1 = false;                               // nothing owned below: pass 2 from the root
+                    lvl = H;
+                    node = 0;
+                    continue;
+                }
+            } else {
+                // S6 with ownership: MINDIST <= pd, unvisited leaves below, owned at level 2
+                const int c_min = visited + 1 < (int)ix.L ? ((visited + 1) >> ((lvl - 1) * LOGF)) - base : F;
+                const int lo_b = min(max(c_min - lane * V, 0), V);
+                unsigned el = mine & ~((1u << lo_b) - 1u);
+#pragma unroll
+                for (int t = 0; t < V; ++t) el &= ~((unsigned)!(md[t] <= pd) << t);
+                const unsigned bal = __ballot_sync(FULL, el != 0);
+                if (bal) {
+                    const int src = __ffs(bal) - 1;
+                    c = src * V + (__ffs(__shfl_sync(FULL, el, src)) - 1);
+                }
+            }
+            if (c < F) {
+                node = base + c;
+                if (--lvl == 0 && pass1) {
+#pragma unroll
+                    for (int t = 0; t < V; ++t) p1md[lane * V + t] = md[t];
+                    if (lane == 0) ws.cache_node[0] = base >> LOGF;
+                    __syncwarp();
+                }
+            } else {                                             // S7 backtrack (R9)
+                if (lvl == H) break;
+                visited = max_leaf(ix, lvl, node);
+                node /= F;
+                ++lvl;
+            }
+        } else {
+            const int j = node;
+            bool changed = false;
+            const bool pre = !pass1 && (j >> LOGF) == ws.cache_node[0] && p1md[j & (F - 1)] < 0.f;
+            if (!pre) changed = scan_leaf<D, V, KS, ST>(ix, j, q, lane, T, k, thr, S, ws.scratch, ws.pf);
+            pd = fminf(pd, key_dist(thr));
+            if (pd < published) {
+                if (lane == 0) publish_pd(g, pd);
+                published = pd;
+            }
+            if (pass1) {                                         // best-first inside N* (R25)
+                const int b1 = j & ~(F - 1);
+                if (lane == 0) p1md[j - b1] = -1.f;
+                __syncwarp();
+                pd = fminf(pd, shared_pd(g));                    // the other parts' progress
+                u64 best = ~0ull;
+#pragma unroll
+                for (int t = 0; t < V; ++t) {
+                    const int cc = lane * V + t;
+                    const float v = p1md[cc];
+                    const u64 kk = make_key(v, cc);
+                    if (v >= 0.f && b1 + cc < L && kk < best) best = kk;
+                }
+                best = warp_min_u64(best);
+                if (best != ~0ull && key_dist(best) <= pd) {
+                    node = b1 + (int)(best & 0xffffffffu);
+                    continue;
+                }
+                pass1 = false;
+                lvl = H;
+                node = 0;
+                continue;
+            }
+            visited = j;
+            if (j == L - 1) break;
+            if (changed && ((j + 1) >> LOGF) == (j >> LOGF)) {
+                node = j + 1;                                    // right sibling in the same (owned) node
+            } else {
+                node = j / F;                                    // parent link
+                lvl = 1;
+            }
+        }
+    }
+    T.store(k, lane, oi, od);
+}
+
+// One warp per (query, part) task; with `queue` the grid is persistent and
+// warps take tasks t = 0, 1, ... from an atomic counter: query order[t / parts]
+// (the closest-leaf order when the batch was reordered), part t % parts.
+template <int D, int V, int KS, bool ST, bool SPH, bool NODE>
 __global__ void __launch_bounds__(WARPS_PER_CTA * 32, MinBlocks<D>::value)
 psb_split_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, int parts, int k,
                  int32_t *__restrict__ part_ids, float *__restrict__ part_dists, float *__restrict__ gpd,
-                 uint32_t variant)
+                 uint32_t variant, unsigned long long *__restrict__ queue, const int32_t *__restrict__ order)
 {
     extern __shared__ __align__(16) unsigned char smem[];
     const int lane = threadIdx.x & 31;
-    const int64_t w = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
-    if (w >= nq * parts) return;
     WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);
     ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) ? PF_NEXT : 0u) | ((variant & PSB_VAR_PREFETCH_IDS) ? PF_IDS : 0u) |
             ((variant & PSB_VAR_P1_INDEX_TIE) ? PF_P1_INDEX_TIE : 0u) |
             ((variant & PSB_VAR_KTH_MAXDIST) || ix.irregular ? PF_KTH_RULE : 0u);
-    psb_part_query<D, V, KS, ST, SPH>(ix, queries, w / parts, (int)(w % parts), parts, k, part_ids, part_dists, gpd, ws,
-                                 !(variant & PSB_VAR_NOCACHE), !(variant & PSB_VAR_NOMAXDIST), lane);
+    const int64_t tasks = nq * parts;
+    int64_t t = (int64_t)blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
+    while (true) {
+        if (queue) {
+            unsigned long long v = 0;
+            if (lane == 0) v = atomicAdd(queue, 1ull);
+            t = (int64_t)__shfl_sync(FULL, v, 0);
+        }
+        if (t >= tasks) break;
+        const int64_t qpos = t / parts;
+        const int64_t qi = order ? (int64_t)__ldg(order + qpos) : qpos;
+        if constexpr (NODE)
+            psb_node_query<D, V, KS, ST, SPH>(ix, queries, qi, (int)(t % parts), parts, k, part_ids, part_dists, gpd,
+                                              ws, !(variant & PSB_VAR_NOCACHE), !(variant & PSB_VAR_NOMAXDIST), lane);
+        else
+            psb_range_query<D, V, KS, ST, SPH>(ix, queries, qi, (int)(t % parts), parts, k, part_ids, part_dists, gpd,
+                                               ws, !(variant & PSB_VAR_NOCACHE), !(variant & PSB_VAR_NOMAXDIST), lane);
+        if (!queue) break;
+    }
 }
 
 template <int D, int V, int KS>
@@ -628,34 +805,6 @@ static int launch_tree_t(int algo, const DevIndex &ix0, const float *queries, in
         e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return report_cuda(e, "cudaFuncSetAttribute");
     }
-    if (parts > 1 && algo == PSB_ALGO_PSB && !counting && KS != 0) {
-        // latency mode: q*parts warps, shared pd per query, then a filtered merge
-        auto sk = ix.sphere ? psb_split_kernel<D, V, KS, false, true> : psb_split_kernel<D, V, KS, false, false>;
-        if (smem > 48 * 1024) {
-            e = cudaFuncSetAttribute(sk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-            if (e != cudaSuccess) return report_cuda(e, "cudaFuncSetAttribute");
-        }
-        int32_t *pi = nullptr;
-        float *pdist = nullptr, *gpd = nullptr;
-        const size_t cnt = (size_t)nq * parts * k;
-        if ((e = cudaMallocFromPoolAsync((void **)&pi, cnt * 4, pool, st)) != cudaSuccess ||
-            (e = cudaMallocFromPoolAsync((void **)&pdist, cnt * 4, pool, st)) != cudaSuccess ||
-            (e = cudaMallocFromPoolAsync((void **)&gpd, (size_t)nq * 4, pool, st)) != cudaSuccess) {
-            if (pi) cudaFreeAsync(pi, st);
-            if (pdist) cudaFreeAsync(pdist, st);
-            return report_cuda(e, "cudaMallocFromPoolAsync (split scratch)");
-        }
-        init_shared_pd(gpd, nq, st);                            // +inf per query
-        const int64_t warps = nq * parts;
-        sk<<<(unsigned)((warps + WARPS_PER_CTA - 1) / WARPS_PER_CTA), WARPS_PER_CTA * 32, smem, st>>>(
-            ix, queries, nq, parts, k, pi, pdist, gpd, variant);
-        int rc = report_cuda(cudaGetLastError(), "split kernel launch");
-        if (rc == PSB_OK) rc = launch_merge_parts(pi, pdist, gpd, parts, nq, k, oi, od, st);
-        cudaFreeAsync(pi, st);
-        cudaFreeAsync(pdist, st);
-        cudaFreeAsync(gpd, st);
-        return rc;
-    }
     // Batch scheduling: process the queries in the order of their closest leaf
     // (knn_order.cu) so concurrent warps share leaves in L1/L2. Rows are written
     // to their input positions, so results are unchanged.
@@ -680,6 +829,56 @@ static int launch_tree_t(int algo, const DevIndex &ix0, const float *queries, in
             cudaFreeAsync(order, st);
             return rc;
         }
+    }
+    if (parts > 1 && algo == PSB_ALGO_PSB && !counting && KS != 0) {
+        // split mode: q*parts (query, part) tasks, shared pd per query, then a filtered merge
+        // whole interleaved level-1 nodes when the (query, part) tasks fill the GPU
+        // (a batch's tail), contiguous leaf ranges otherwise (single-query latency)
+        using SK = void (*)(DevIndex, const float *, int64_t, int, int, int32_t *, float *, float *, uint32_t,
+                            unsigned long long *, const int32_t *);
+        SK skn = ix.sphere ? psb_split_kernel<D, V, KS, false, true, true> : psb_split_kernel<D, V, KS, false, false, true>;
+        SK skr = ix.sphere ? psb_split_kernel<D, V, KS, false, true, false> : psb_split_kernel<D, V, KS, false, false, false>;
+        int sper = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&sper, skn, WARPS_PER_CTA * 32, smem) != cudaSuccess || sper < 1)
+            sper = 1;
+        cudaGetLastError();
+        const int64_t tasks = nq * parts;
+        const int64_t resident = (int64_t)sper * ix.sm_count * WARPS_PER_CTA;
+        const SK sk = tasks >= resident ? skn : skr;
+        if (smem > 48 * 1024 && (e = cudaFuncSetAttribute(sk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
+                                    cudaSuccess) {
+            if (order) cudaFreeAsync(order, st);
+            return report_cuda(e, "cudaFuncSetAttribute");
+        }
+        int32_t *pi = nullptr;
+        float *pdist = nullptr, *gpd = nullptr;
+        unsigned long long *squeue = nullptr;
+        const size_t cnt = (size_t)nq * parts * k;
+        if ((e = cudaMallocFromPoolAsync((void **)&pi, cnt * 4, pool, st)) != cudaSuccess ||
+            (e = cudaMallocFromPoolAsync((void **)&pdist, cnt * 4, pool, st)) != cudaSuccess ||
+            (e = cudaMallocFromPoolAsync((void **)&gpd, (size_t)nq * 4, pool, st)) != cudaSuccess ||
+            (e = cudaMallocFromPoolAsync((void **)&squeue, sizeof(unsigned long long), pool, st)) != cudaSuccess) {
+            if (pi) cudaFreeAsync(pi, st);
+            if (pdist) cudaFreeAsync(pdist, st);
+            if (gpd) cudaFreeAsync(gpd, st);
+            if (order) cudaFreeAsync(order, st);
+            return report_cuda(e, "cudaMallocFromPoolAsync (split scratch)");
+        }
+        init_shared_pd(gpd, nq, st);                            // +inf per query
+        cudaMemsetAsync(squeue, 0, sizeof(unsigned long long), st);
+        int64_t sblocks = (tasks + WARPS_PER_CTA - 1) / WARPS_PER_CTA;
+        const bool persistent = sblocks * WARPS_PER_CTA > resident;
+        if (persistent) sblocks = resident / WARPS_PER_CTA;
+        sk<<<(unsigned)sblocks, WARPS_PER_CTA * 32, smem, st>>>(ix, queries, nq, parts, k, pi, pdist, gpd, variant,
+                                                                 persistent ? squeue : nullptr, order);
+        int rc = report_cuda(cudaGetLastError(), "split kernel launch");
+        if (rc == PSB_OK) rc = launch_merge_parts(pi, pdist, gpd, parts, nq, k, oi, od, st);
+        cudaFreeAsync(pi, st);
+        cudaFreeAsync(pdist, st);
+        cudaFreeAsync(gpd, st);
+        cudaFreeAsync(squeue, st);
+        if (order) cudaFreeAsync(order, st);
+        return rc;
     }
     // More queries than resident warps: persistent grid + atomic query queue.
     int per_sm = 0;

@@ -181,6 +181,10 @@ def test_c4_full_batch_all_rows():
     for algo in ("psb", "bnb"):
         assert_same(run(idx, qs, cfg.k, algo), exp, f"C4 {algo} (full batch)")
     assert_same(run(idx, qs[:200], cfg.k, "brute"), (exp[0][:200], exp[1][:200]), "C4 brute")
+    # the batch split into interleaved-node parts (auto: 2-8 parts per query)
+    si, sd = _psb().psb_knn_split(idx, torch.from_numpy(qs).cuda(), cfg.k, parts=0)
+    torch.cuda.synchronize()
+    assert_same((si.cpu().numpy(), sd.cpu().numpy()), exp, "C4 psb split (full batch)")
     idx.free()
 
 
@@ -412,10 +416,13 @@ def test_gpu_bulk_load_matches_host_loader(case):
     host.free()
 
 
-@pytest.mark.parametrize("nq,parts", [(1, 0), (1, 7), (3, 64), (64, 0), (1000, 2), (200, 1)])
+@pytest.mark.parametrize("nq,parts", [(1, 0), (1, 7), (3, 64), (64, 0), (1000, 2), (200, 1),
+                                      (5000, 2), (8000, 5), (9000, 8)])
 def test_split_latency_mode(c2, nq, parts):
-    """psb_knn_split (each query's leaves over `parts` warps, shared pruning
-    distance, filtered merge) returns exactly psb_knn's rows."""
+    """psb_knn_split (each query over `parts` warps, shared pruning distance,
+    filtered merge) returns exactly psb_knn's rows, in both ownership modes:
+    contiguous leaf ranges (few tasks) and interleaved level-1 nodes (the last
+    three cases fill the GPU with (query, part) tasks)."""
     psb = _psb()
     cfg, pts, qs, idx, exp = c2
     sl = slice(100, 100 + nq)
