@@ -61,7 +61,8 @@ def parse():
                     help="data mode on ONE GPU: run rank 0's local step of a P-way data-sharded job")
     ap.add_argument("--exchange", default="p2p", choices=["p2p", "nccl"],
                     help="data mode, N>1: merge straight from peer memory (psb_exchange) or NCCL all-gather + merge")
-    ap.add_argument("--algo", default="psb", choices=["psb", "bnb", "brute"])
+    ap.add_argument("--algo", default="psb", choices=["psb", "psb_split", "bnb", "brute"],
+                    help="psb_split: psb_knn_split with the library's automatic part count")
     ap.add_argument("--variant", type=int, default=0)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -273,6 +274,13 @@ def roofline(algo, idx, q, k, alg_bytes, kern_s, prof_cfg, l2_peak):
                 "peak_source": "148 SMs x 128 FP32 lanes x sm_max_mhz: packed FADD2/FFMA2 pairs issue at one "
                                "per 2 cycles per SMSP (ncu: fma pipe busy 2 cycles per packed instruction; "
                                "DESIGN.md §6)"}
+    elif alg_bytes is None:                   # split mode: ncu's L2 bytes of the split kernel
+        l2b = traffic_from_profiles(prof_cfg, algo, "l2_bytes_per_launch") or 0.0
+        a = l2b / kern_s / 1e9
+        prim = {"bound": "l2", "achieved": a, "peak": l2_peak, "unit": "GB/s", "frac": a / l2_peak,
+                "l2_bytes_per_launch": l2b, "note": "split mode has no per-part traversal counters: "
+                "achieved = ncu lts bytes of psb_split_kernel (profiles/traffic.json) / live launch time",
+                "peak_source": "measured in this run: psb_probe_l2_read (64 MiB L2-resident, ld.global.cg)"}
     else:
         a = alg_bytes / kern_s / 1e9
         prim = {"bound": "l2", "achieved": a, "peak": l2_peak, "unit": "GB/s", "frac": a / l2_peak,
@@ -345,7 +353,8 @@ def main():
     cfg = W.config(args.config)
     q = args.queries or cfg.q
     k = cfg.k
-    algo = {"psb": psb.PSB_ALGO_PSB, "bnb": psb.PSB_ALGO_BNB, "brute": psb.PSB_ALGO_BRUTE}[args.algo]
+    algo = {"psb": psb.PSB_ALGO_PSB, "psb_split": psb.PSB_ALGO_PSB, "bnb": psb.PSB_ALGO_BNB,
+            "brute": psb.PSB_ALGO_BRUTE}[args.algo]
     weak = args.mode == "query" and args.weak
     if args.mode == "query":
         # replicated index; strong scaling: rank r answers slice r of the fixed
@@ -375,6 +384,10 @@ def main():
         alg_bytes = idx.leaves * idx.fanout * (idx.d * 4) * ql + ql * (4 * idx.d + 8 * k)
         stats_sum = None
         in_batch = None
+    elif args.algo == "psb_split":            # no per-part counters: the roofline uses ncu's L2 bytes
+        alg_bytes = None
+        stats_sum = None
+        in_batch = None
     else:
         _, _, st = psb.psb_knn_stats(idx, qd, k, algo=algo, variant=args.variant, out=(out_i, out_d))
         stn = st.cpu().numpy()
@@ -391,8 +404,10 @@ def main():
                                   "took / finished the query), counting-kernel instantiation"}
 
     def local_knn(qq, kk):
-        return psb.psb_knn_ex(idx, qq, kk, algo=algo, variant=args.variant,
-                              out=(out_i, out_d) if qq.shape[0] == ql else None)
+        o = (out_i, out_d) if qq.shape[0] == ql else None
+        if args.algo == "psb_split":
+            return psb.psb_knn_split(idx, qq, kk, parts=0, out=o)
+        return psb.psb_knn_ex(idx, qq, kk, algo=algo, variant=args.variant, out=o)
 
     ex = None
     chunks = max(1, args.chunks)
@@ -446,7 +461,8 @@ def main():
     # as its own workload (tools/prof_one.py C5 = slab 0 of 8 -> "C5slab")
     prof_cfg = args.config + ("slab" if args.mode == "data" and world == 1 and (args.slab or 1) == 8 else "")
     roof = roofline(args.algo, idx, ql, k, alg_bytes, kern_s, prof_cfg, l2_peak)
-    roof["kernel"] = {"psb": "psb_kernel", "bnb": "bnb_kernel", "brute": "brute_kernel+merge_kernel"}[args.algo]
+    roof["kernel"] = {"psb": "psb_kernel", "psb_split": "psb_split_kernel", "bnb": "bnb_kernel",
+                      "brute": "brute_smem_kernel"}[args.algo]
     if stats_sum is not None:
         roof["counters_per_query"] = {"node_fetches": stats_sum[0] / ql, "leaf_scans": stats_sum[1] / ql,
                                       "id_loads": stats_sum[2] / ql, "cache_hits": stats_sum[3] / ql,
@@ -456,6 +472,12 @@ def main():
     if not args.no_extras:
         # e2e through the public API with HOST (pinned) buffers: H2D + kernel + D2H each step
         hq = torch.from_numpy(qs).pin_memory()
+
+        def local_e2e(x, oi, od):
+            if args.algo == "psb_split":
+                return psb.psb_knn_split(idx, x, k, parts=0, out=(oi, od))
+            return psb.psb_knn_ex(idx, x, k, algo=algo, variant=args.variant, out=(oi, od))
+
         hi = torch.empty((ql, k), dtype=torch.int32, pin_memory=True)
         hd = torch.empty((ql, k), dtype=torch.float32, pin_memory=True)
         e2e_ms = []
@@ -463,7 +485,7 @@ def main():
             flush.fill_(i & 0xFF)
             torch.cuda.synchronize()
             t0 = time.perf_counter()
-            psb.psb_knn_ex(idx, hq, k, algo=algo, variant=args.variant, out=(hi, hd))
+            local_e2e(hq, hi, hd)
             stream.synchronize()
             if i >= max(3, args.warmup):
                 e2e_ms.append((time.perf_counter() - t0) * 1e3)
@@ -497,7 +519,7 @@ def main():
                     "queries": n_lat}
 
         lats = {
-            args.algo: lat_of(lambda x: psb.psb_knn_ex(idx, x, k, algo=algo, variant=args.variant, out=(h1i, h1d)), nl),
+            args.algo: lat_of(lambda x: local_e2e(x, h1i, h1d), nl),
             "psb_split": lat_of(lambda x: psb.psb_knn_split(idx, x, k, parts=0, out=(h1i, h1d)), nl),
             "bnb": lat_of(lambda x: psb.psb_knn_ex(idx, x, k, algo=psb.PSB_ALGO_BNB, out=(h1i, h1d)), nl),
             "brute": lat_of(lambda x: psb.psb_knn_ex(idx, x, k, algo=psb.PSB_ALGO_BRUTE, out=(h1i, h1d)),

@@ -399,21 +399,24 @@ int psb_knn_split(const psb_index *ix, const float *queries, int64_t q, int32_t 
     if (ix && parts == 0) {
         // auto (DESIGN.md §6 "split mode"):
         //  - few queries (<= 1/4 of the resident warps): latency mode, about 16
-        //    warps per SM in total, at least 16 leaves per part;
+        //    warps per SM in total, at least 16 leaves per part, when the
+        //    estimated leaves per query (below) reach 16;
         //  - a batch that fills the GPU less than 4 times over, of queries that
         //    touch many leaves: 2-8 parts per query against the batch's tail. The
         //    work per query is estimated by the classic uniform-data cost model
         //    (1 + (k'/F)^(1/d))^d leaves (k' = min(k, F)): >= 64 splits;
         //  - otherwise 1 (plain psb_knn).
         const int64_t resident = (int64_t)ix->sm_count * 32;
+        const double kf = (double)(k < ix->F ? k : ix->F) / ix->F;
+        const double work = std::pow(1.0 + std::pow(kf, 1.0 / ix->d), (double)ix->d);
         int64_t p = 1;
         if (q * 4 <= resident) {
-            p = q > 0 ? (int64_t)ix->sm_count * 16 / q : 1;
-            const int64_t pmax = ix->L / 16;
-            if (p > pmax) p = pmax;
+            if (work >= 16.0) {                   // else one warp is faster than the split's overhead
+                p = q > 0 ? (int64_t)ix->sm_count * 16 / q : 1;
+                const int64_t pmax = ix->L / 16;
+                if (p > pmax) p = pmax;
+            }
         } else if (q < 4 * resident) {
-            const double kf = (double)(k < ix->F ? k : ix->F) / ix->F;
-            const double work = std::pow(1.0 + std::pow(kf, 1.0 / ix->d), (double)ix->d);
             if (work >= 64.0) {
                 p = 12 * resident / q;
                 p = p < 2 ? 2 : (p > 8 ? 8 : p);

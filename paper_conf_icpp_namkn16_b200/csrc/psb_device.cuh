@@ -28,6 +28,11 @@ typedef unsigned long long u64;
 #ifndef PSB_INSERT_MAX_KS1
 #define PSB_INSERT_MAX_KS1 1
 #endif
+// Sizes of the candidate sorting network in TopK::offer (code size vs work):
+// 3 = 8 / 16 / 32 candidates, 2 = 8 / 32, 1 = 32 only.
+#ifndef PSB_MERGE_SIZES
+#define PSB_MERGE_SIZES 3
+#endif
 constexpr unsigned FULL = 0xffffffffu;
 enum : unsigned { PF_NEXT = 1u, PF_IDS = 2u, PF_P1_INDEX_TIE = 4u, PF_KTH_RULE = 8u };   // per-launch traversal flags
 // (dist, id) packed as one u64 key: for dist >= +0 the IEEE bit pattern orders
@@ -503,9 +508,16 @@ struct TopK {
             const int n = min(m - r, 32);
             const u64 c = lane < n ? scratch[lane] : ~0ull;
             __syncwarp();
+#if PSB_MERGE_SIZES == 1
+            merge32<32>(c, lane);
+#elif PSB_MERGE_SIZES == 2
+            if (n <= 8) merge32<8>(c, lane);
+            else merge32<32>(c, lane);
+#else
             if (n <= 8) merge32<8>(c, lane);
             else if (n <= 16) merge32<16>(c, lane);
             else merge32<32>(c, lane);
+#endif
         }
         thr = kth(k);
         return m;

@@ -1,5 +1,5 @@
 """One warm-up launch then one profiled launch of a tree kernel (for ncu -k/-c). Dev aid.
-usage: prof_one.py CONFIG ALGO(psb|bnb|brute) [VARIANT]"""
+usage: prof_one.py CONFIG ALGO(psb|psb_split|bnb|brute) [VARIANT]"""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
@@ -17,8 +17,11 @@ else:
     pts = cfg.points()
 qd = torch.from_numpy(cfg.queries()).cuda()
 idx = psb.psb_build(pts, cfg.fanout)
-a = {"psb": 0, "bnb": 1, "brute": 2}[algo]
+a = {"psb": 0, "psb_split": 0, "bnb": 1, "brute": 2}[algo]
 for _ in range(2):
-    psb.psb_knn_ex(idx, qd, cfg.k, algo=a, variant=var)
+    if algo == "psb_split":
+        psb.psb_knn_split(idx, qd, cfg.k, parts=0)
+    else:
+        psb.psb_knn_ex(idx, qd, cfg.k, algo=a, variant=var)
 torch.cuda.synchronize()
 idx.free()
