@@ -1,6 +1,4 @@
-O=gpurun_out/r02ba; mkdir -p $O
-nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > $O/smi.txt
-timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.txt 2>&1
-timeout 1500 python -m pytest tests -m gpu -x -q > $O/gputests.txt 2>&1
-timeout 600 python bench.py > $O/bench_C3.json 2> $O/bench_C3.err
-tail -3 $O/gputests.txt; cat $O/smoke.txt; head -c 400 $O/bench_C3.json
+O=gpurun_out/r02bf; mkdir -p $O
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:psb_kernel -s 1 -c 1 -o $O/c5_psb python tools/prof_one.py C5 psb > $O/ncu_c5.log 2>&1
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:bnb_kernel -s 1 -c 1 -o $O/c5_bnb python tools/prof_one.py C5 bnb > $O/ncu_c5b.log 2>&1
+tail -1 $O/ncu_c5.log $O/ncu_c5b.log
