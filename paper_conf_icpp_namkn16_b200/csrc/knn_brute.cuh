@@ -9,6 +9,9 @@
 // (|x|^2 - 2x.y + |y|^2 rounds differently and would break bit-exactness).
 #include <cuda_runtime.h>
 
+#include <algorithm>
+#include <cstdlib>
+
 #include "psb_device.cuh"
 #include "psb_launch.h"
 
@@ -240,13 +243,34 @@ static int launch_brute_smem(const DevIndex &ix, const float *queries, int64_t n
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, BS_WARPS * 32, smem) != cudaSuccess || per_sm < 1)
         per_sm = 1;
     cudaGetLastError();
-    // split the leaves into S chunks so that the grid covers every resident CTA
-    // slot about twice; chunks never shorter than 8 leaves
-    int64_t S = ((int64_t)sm_count * per_sm * 2 + blocks_q - 1) / blocks_q;
-    const int64_t smax = (ix.L + 7) / 8;
-    if (S > smax) S = smax;
-    if (S > 1024) S = 1024;
-    if (S < 1) S = 1;
+    // Split the leaves into S chunks. A small batch (too few CTAs to fill the GPU
+    // twice with chunks of >= 2048 leaves: single-query latency) gets about two
+    // CTAs per slot, chunks down to 8 leaves. A large batch gets chunks of >= 2048
+    // leaves, and since every CTA then does the same work, the launch takes
+    // ceil(blocks / slots) waves of equal length: take the smallest S whose waves
+    // are >= 90 % full on average (at least two waves' worth of CTAs), else the
+    // fullest up to S = 64. More chunks cost partial lists and a longer merge, so
+    // the threshold is not higher. C4 (313 query blocks on 296 slots): round 1's
+    // "two CTAs per slot" rule gave S = 2, 2.11 waves with a third wave of 34 CTAs
+    // (22 % achieved occupancy), 317 ms; S = 6 takes 279 ms, S = 12 286 ms,
+    // S = 24 293 ms (profiles/r02bh).
+    const int64_t slots = (int64_t)sm_count * per_sm;
+    const int64_t smax_big = std::min<int64_t>(ix.L / 2048, 64);
+    const int64_t smax = std::max<int64_t>(1, std::min<int64_t>((ix.L + 7) / 8, 1024));
+    int64_t S = 1;
+    if (blocks_q * smax_big < 2 * slots) {
+        S = std::min<int64_t>(smax, (2 * slots + blocks_q - 1) / blocks_q);
+    } else {
+        double best = -1.0;
+        for (int64_t c = 1; c <= smax_big; ++c) {
+            const int64_t blocks = blocks_q * c;
+            const int64_t waves = (blocks + slots - 1) / slots;
+            const double eff = (double)blocks / ((double)waves * slots);
+            if (blocks >= 2 * slots && eff >= 0.90) { S = c; break; }
+            if (eff > best + 1e-9) { S = c; best = eff; }
+        }
+    }
+    if (const char *ev = getenv("PSB_BRUTE_CHUNKS")) S = std::max<int64_t>(1, std::min<int64_t>(atoll(ev), smax));   // A/B
     const int64_t per = (ix.L + S - 1) / S;
     S = (ix.L + per - 1) / per;
     int32_t *pi = oi;
