@@ -44,7 +44,9 @@ for sigma in [float(s) for s in sys.argv[1:]] or [10, 40, 160, 640, 2560, 10240]
     for name, a in (("psb", 0), ("bnb", 1), ("brute", 2)):
         res[name] = psb.psb_knn_ex(idx, qd, k, algo=a)
         ms[name] = batch_ms(lambda: psb.psb_knn_ex(idx, qd, k, algo=a))
-    same = all(torch.equal(res["psb"][j], res[o][j]) for o in ("bnb", "brute") for j in (0, 1))
+    res["psb_split"] = psb.psb_knn_split(idx, qd, k, parts=0)          # auto parts (tail splitting)
+    ms["psb_split"] = batch_ms(lambda: psb.psb_knn_split(idx, qd, k, parts=0))
+    same = all(torch.equal(res["psb"][j], res[o][j]) for o in ("bnb", "brute", "psb_split") for j in (0, 1))
     ei, ed = oracle.knn_bruteforce(pts, qs[:16], k)
     ok = bool(np.array_equal(res["psb"][0][:16].cpu().numpy(), ei) and
               np.array_equal(res["psb"][1][:16].cpu().numpy().view(np.uint32), ed.view(np.uint32)))
