@@ -22,11 +22,14 @@
  *  - Layouts: points[n][d], queries[q][d] fp32 row-major; out_ids[q][k] int32,
  *    out_dists[q][k] fp32, row-major.
  *  - Queries and outputs may be CUDA device pointers on the index's device or
- *    host memory. Host queries and pageable host outputs are staged through
- *    stream-ordered device scratch with cudaMemcpyAsync on `stream`; pinned
- *    (page-locked, hence device-mapped) host outputs are written directly by
- *    the kernels, row by row as queries finish (zero-copy). Either way the
- *    results are in host memory once the stream reaches the end of the call
+ *    host memory. Pinned (page-locked, hence device-mapped) host buffers are
+ *    used in place by the kernels (zero-copy): result rows are written row by
+ *    row as queries finish, and the one-warp-per-query traversals read each
+ *    query's d floats over the host link (split mode and brute force, where many
+ *    warps read each query, stage pinned queries with one copy). Pageable host
+ *    queries and outputs are staged through stream-ordered device scratch with
+ *    cudaMemcpyAsync on `stream`. Either way
+ *    the results are in host memory once the stream reaches the end of the call
  *    (psb_build: points may be host or device memory).
  *  - Query calls are asynchronous on `stream` (a cudaStream_t; NULL = legacy
  *    default stream). Argument errors are returned synchronously without

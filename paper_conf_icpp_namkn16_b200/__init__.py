@@ -104,14 +104,25 @@ def psb_version() -> str:
     return _lib.psb_version().decode()
 
 
+_TORCH = None
+
+
 def _torch():
-    import torch
-    return torch
+    global _TORCH
+    if _TORCH is None:
+        import torch
+        _TORCH = torch
+    return _TORCH
 
 
-def _stream_handle(stream) -> int:
-    torch = _torch()
+def _stream_handle(stream, device: int | None = None) -> int:
+    """cudaStream_t of `stream` (None: torch's current stream on `device`). The raw
+    getter avoids building a Stream object: a one-query call is host-latency bound."""
     if stream is None:
+        torch = _torch()
+        raw = getattr(torch._C, "_cuda_getCurrentRawStream", None)
+        if raw is not None:
+            return int(raw(torch.cuda.current_device() if device is None else device))
         stream = torch.cuda.current_stream()
     return int(stream.cuda_stream) if hasattr(stream, "cuda_stream") else int(stream)
 
@@ -177,53 +188,57 @@ def psb_build(points, fanout: int) -> Index:
     return Index(h)
 
 
-def _check_out(out, q: int, k: int, device):
-    """out = (ids, dists): int32 / float32 [q, k] C-contiguous tensors, on `device`
-    or in host memory."""
+def _check_out(out, q: int, k: int, device: int):
+    """out = (ids, dists): int32 / float32 [q, k] C-contiguous tensors, on CUDA
+    device `device` or in host memory."""
     torch = _torch()
     ids, dists = out
     for t, dt, name in ((ids, torch.int32, "ids"), (dists, torch.float32, "dists")):
-        if t.dtype != dt or tuple(t.shape) != (q, k) or not t.is_contiguous():
+        if t.dtype is not dt or t.shape != (q, k) or not t.is_contiguous():
             raise ValueError(f"out {name} must be a contiguous {dt} [{q}, {k}] tensor")
-        if t.is_cuda and t.device != device:
-            raise ValueError(f"out {name} is on {t.device}, the index on {device}")
+        if t.is_cuda and t.get_device() != device:
+            raise ValueError(f"out {name} is on {t.device}, the index on cuda:{device}")
 
 
 def _query_buffers(index: Index, queries, k: int, out):
     """Queries: float32 [q, d] tensor on the index's device, or a CPU tensor
-    (pinned for asynchronous copies) — then the library stages it on the stream.
+    (pinned: read in place by the kernels; pageable: staged by the library).
     Outputs default to the queries' device (CPU outputs are pinned)."""
     torch = _torch()
-    if not (queries.dtype == torch.float32 and queries.dim() == 2 and queries.shape[1] == index.d):
+    if queries.dtype is not torch.float32 or queries.dim() != 2 or queries.shape[1] != index.d:
         raise ValueError(f"queries must be a float32 [q, {index.d}] tensor")
-    queries = queries.contiguous()
+    if not queries.is_contiguous():
+        queries = queries.contiguous()
     q = queries.shape[0]
-    dev = torch.device("cuda", index.device)
-    if queries.is_cuda and queries.device != dev:
-        raise ValueError(f"queries are on {queries.device}, the index on {dev}")
+    if queries.is_cuda and queries.get_device() != index.device:
+        raise ValueError(f"queries are on {queries.device}, the index on cuda:{index.device}")
     if out is None:
         pin = not queries.is_cuda
         ids = torch.empty((q, k), dtype=torch.int32, device=queries.device, pin_memory=pin)
         dists = torch.empty((q, k), dtype=torch.float32, device=queries.device, pin_memory=pin)
     else:
-        _check_out(out, q, k, dev)
+        _check_out(out, q, k, index.device)
         ids, dists = out
     return queries, q, ids, dists
 
 
 def _host_sync(stream, *tensors):
     """The C ABI is asynchronous and keeps no reference to its buffers. Host
-    tensors (queries read by a stream-ordered copy, outputs written by the
-    kernels) would otherwise be returned while the device still uses them, and a
-    temporary pinned input could be recycled by torch's caching host allocator:
+    tensors (queries read in place or by a stream-ordered copy, outputs written by
+    the kernels) would otherwise be returned while the device still uses them, and
+    a temporary pinned input could be recycled by torch's caching host allocator:
     with any host tensor, the call waits for its stream before returning."""
-    if any(not t.is_cuda for t in tensors):
-        torch = _torch()
-        s = stream if stream is not None else torch.cuda.current_stream()
-        if hasattr(s, "synchronize"):
-            s.synchronize()
-        else:
-            torch.cuda.ExternalStream(int(s)).synchronize()
+    for t in tensors:
+        if not t.is_cuda:
+            break
+    else:
+        return
+    torch = _torch()
+    s = stream if stream is not None else torch.cuda.current_stream()
+    if hasattr(s, "synchronize"):
+        s.synchronize()
+    else:
+        torch.cuda.ExternalStream(int(s)).synchronize()
 
 
 def psb_knn_ex(index: Index, queries, k: int, algo: int = PSB_ALGO_PSB, variant: int = 0,
@@ -232,7 +247,7 @@ def psb_knn_ex(index: Index, queries, k: int, algo: int = PSB_ALGO_PSB, variant:
     tensors; waits for the stream when a tensor is in host memory. Returns (ids, dists)."""
     queries, q, ids, dists = _query_buffers(index, queries, k, out)
     _check(_lib.psb_knn_ex(index.handle, queries.data_ptr(), q, k, ids.data_ptr(), dists.data_ptr(),
-                           _stream_handle(stream), algo, variant), "psb_knn_ex")
+                           _stream_handle(stream, index.device), algo, variant), "psb_knn_ex")
     _host_sync(stream, queries, ids, dists)
     return ids, dists
 
@@ -396,7 +411,7 @@ class Exchange:
         if out is None:
             return (torch.empty((rows, self.k), dtype=torch.int32, device="cuda"),
                     torch.empty((rows, self.k), dtype=torch.float32, device="cuda"))
-        _check_out(out, rows, self.k, torch.device("cuda", torch.cuda.current_device()))
+        _check_out(out, rows, self.k, torch.cuda.current_device())
         return out
 
     def merge(self, row0: int, rows: int, stream=None, out=None):

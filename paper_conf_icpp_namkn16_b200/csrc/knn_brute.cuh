@@ -239,10 +239,8 @@ static int launch_brute_smem(const DevIndex &ix, const float *queries, int64_t n
     if (smem > 48 * 1024 && (e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
                                 cudaSuccess)
         return report_cuda(e, "cudaFuncSetAttribute (brute smem)");
-    int per_sm = 1;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, BS_WARPS * 32, smem) != cudaSuccess || per_sm < 1)
-        per_sm = 1;
-    cudaGetLastError();
+    int per_sm = cached_occupancy((const void *)kern, BS_WARPS * 32, smem);
+    if (per_sm < 1) per_sm = 1;
     // Split the leaves into S chunks. A small batch (too few CTAs to fill the GPU
     // twice with chunks of >= 2048 leaves: single-query latency) gets about two
     // CTAs per slot, chunks down to 8 leaves. A large batch gets chunks of >= 2048

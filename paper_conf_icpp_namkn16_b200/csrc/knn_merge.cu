@@ -97,15 +97,16 @@ merge_parts_kernel(const int32_t *__restrict__ ids, const float *__restrict__ di
     }
 }
 
-__global__ void fill_inf(float *__restrict__ p, int64_t n)
+__global__ void fill_inf(float *__restrict__ p, int64_t n, unsigned long long *__restrict__ queue)
 {
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i < n) p[i] = INFINITY;
+    if (queue && i == 0) *queue = 0ull;
 }
 
-void init_shared_pd(float *gpd, int64_t nq, cudaStream_t st)
+void init_shared_pd(float *gpd, int64_t nq, unsigned long long *queue, cudaStream_t st)
 {
-    fill_inf<<<(unsigned)((nq + 255) / 256), 256, 0, st>>>(gpd, nq);
+    fill_inf<<<(unsigned)((nq + 255) / 256), 256, 0, st>>>(gpd, nq, queue);
 }
 
 // Few parts per query (split batches): one warp per query over its [parts][k]

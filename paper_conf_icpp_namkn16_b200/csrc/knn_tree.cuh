@@ -838,10 +838,8 @@ static int launch_tree_t(int algo, const DevIndex &ix0, const float *queries, in
                             unsigned long long *, const int32_t *);
         SK skn = ix.sphere ? psb_split_kernel<D, V, KS, false, true, true> : psb_split_kernel<D, V, KS, false, false, true>;
         SK skr = ix.sphere ? psb_split_kernel<D, V, KS, false, true, false> : psb_split_kernel<D, V, KS, false, false, false>;
-        int sper = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&sper, skn, WARPS_PER_CTA * 32, smem) != cudaSuccess || sper < 1)
-            sper = 1;
-        cudaGetLastError();
+        int sper = cached_occupancy((const void *)skn, WARPS_PER_CTA * 32, smem);
+        if (sper < 1) sper = 1;
         const int64_t tasks = nq * parts;
         const int64_t resident = (int64_t)sper * ix.sm_count * WARPS_PER_CTA;
         const SK sk = tasks >= resident ? skn : skr;
@@ -850,41 +848,35 @@ static int launch_tree_t(int algo, const DevIndex &ix0, const float *queries, in
             if (order) cudaFreeAsync(order, st);
             return report_cuda(e, "cudaFuncSetAttribute");
         }
-        int32_t *pi = nullptr;
-        float *pdist = nullptr, *gpd = nullptr;
-        unsigned long long *squeue = nullptr;
+        // one scratch allocation: [queue u64][gpd nq][ids cnt][dists cnt]
         const size_t cnt = (size_t)nq * parts * k;
-        if ((e = cudaMallocFromPoolAsync((void **)&pi, cnt * 4, pool, st)) != cudaSuccess ||
-            (e = cudaMallocFromPoolAsync((void **)&pdist, cnt * 4, pool, st)) != cudaSuccess ||
-            (e = cudaMallocFromPoolAsync((void **)&gpd, (size_t)nq * 4, pool, st)) != cudaSuccess ||
-            (e = cudaMallocFromPoolAsync((void **)&squeue, sizeof(unsigned long long), pool, st)) != cudaSuccess) {
-            if (pi) cudaFreeAsync(pi, st);
-            if (pdist) cudaFreeAsync(pdist, st);
-            if (gpd) cudaFreeAsync(gpd, st);
+        const size_t o_gpd = 16, o_ids = (o_gpd + (size_t)nq * 4 + 15) & ~(size_t)15;
+        const size_t o_d = (o_ids + cnt * 4 + 15) & ~(size_t)15;
+        unsigned char *scratch = nullptr;
+        if ((e = cudaMallocFromPoolAsync((void **)&scratch, o_d + cnt * 4, pool, st)) != cudaSuccess) {
             if (order) cudaFreeAsync(order, st);
             return report_cuda(e, "cudaMallocFromPoolAsync (split scratch)");
         }
-        init_shared_pd(gpd, nq, st);                            // +inf per query
-        cudaMemsetAsync(squeue, 0, sizeof(unsigned long long), st);
+        unsigned long long *squeue = reinterpret_cast<unsigned long long *>(scratch);
+        float *gpd = reinterpret_cast<float *>(scratch + o_gpd);
+        int32_t *pi = reinterpret_cast<int32_t *>(scratch + o_ids);
+        float *pdist = reinterpret_cast<float *>(scratch + o_d);
         int64_t sblocks = (tasks + WARPS_PER_CTA - 1) / WARPS_PER_CTA;
         const bool persistent = sblocks * WARPS_PER_CTA > resident;
         if (persistent) sblocks = resident / WARPS_PER_CTA;
+        init_shared_pd(gpd, nq, persistent ? squeue : nullptr, st);   // +inf per query, queue 0
         sk<<<(unsigned)sblocks, WARPS_PER_CTA * 32, smem, st>>>(ix, queries, nq, parts, k, pi, pdist, gpd, variant,
                                                                  persistent ? squeue : nullptr, order);
         int rc = report_cuda(cudaGetLastError(), "split kernel launch");
         if (rc == PSB_OK) rc = launch_merge_parts(pi, pdist, gpd, parts, nq, k, oi, od, st);
-        cudaFreeAsync(pi, st);
-        cudaFreeAsync(pdist, st);
-        cudaFreeAsync(gpd, st);
-        cudaFreeAsync(squeue, st);
+        cudaFreeAsync(scratch, st);
         if (order) cudaFreeAsync(order, st);
         return rc;
     }
     // More queries than resident warps: persistent grid + atomic query queue.
-    int per_sm = 0;
+    const int per_sm = cached_occupancy((const void *)kern, WARPS_PER_CTA * 32, smem);
     unsigned long long *queue = nullptr;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, WARPS_PER_CTA * 32, smem) == cudaSuccess &&
-        per_sm > 0 && blocks > (int64_t)per_sm * ix.sm_count) {
+    if (per_sm > 0 && blocks > (int64_t)per_sm * ix.sm_count) {
         if ((e = cudaMallocFromPoolAsync((void **)&queue, sizeof(unsigned long long), pool, st)) != cudaSuccess) {
             if (order) cudaFreeAsync(order, st);
             return report_cuda(e, "cudaMallocFromPoolAsync (query queue)");

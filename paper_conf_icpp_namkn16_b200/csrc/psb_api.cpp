@@ -8,7 +8,10 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <map>
+#include <mutex>
 #include <new>
+#include <tuple>
 
 #include "psb_internal.h"
 #include "psb_launch.h"
@@ -28,6 +31,28 @@ void psb_set_error(const char *fmt, ...)
 }
 
 namespace psb {
+int cached_occupancy(const void *kern, int threads, size_t smem)
+{
+    static std::mutex mu;
+    static std::map<std::tuple<const void *, int, size_t, int>, int> memo;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const auto key = std::make_tuple(kern, threads, smem, dev);
+    {
+        std::lock_guard<std::mutex> g(mu);
+        auto it = memo.find(key);
+        if (it != memo.end()) return it->second;
+    }
+    int n = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, threads, smem) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;                      // not memoised: a later call may succeed
+    }
+    std::lock_guard<std::mutex> g(mu);
+    memo[key] = n;
+    return n;
+}
+
 int report_cuda(cudaError_t e, const char *what)
 {
     if (e == cudaSuccess) return PSB_OK;
@@ -272,19 +297,23 @@ static bool is_device_ptr(const void *p)
     return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
-// Device address of page-locked (pinned or registered) host memory, mapped into
-// the device's address space; nullptr for pageable memory.
-static void *mapped_host_ptr(void *p)
+// true for device (or managed) memory; otherwise *mapped = the device address of
+// page-locked (pinned or registered) host memory, nullptr for pageable memory.
+static bool ptr_info(const void *p, void **mapped)
 {
+    *mapped = nullptr;
     cudaPointerAttributes a;
     if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
         cudaGetLastError();
-        return nullptr;
+        return false;
     }
-    return a.type == cudaMemoryTypeHost ? a.devicePointer : nullptr;
+    if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) return true;
+    if (a.type == cudaMemoryTypeHost) *mapped = a.devicePointer;
+    return false;
 }
 
-// Launch one algorithm on device buffers; host buffers (pinned or pageable) are
+// Launch one algorithm on device buffers. Host buffers: pinned ones are used in
+// place by the kernels (zero-copy queries and result rows), pageable ones are
 // staged through stream-ordered device scratch with copies on the same stream.
 static int knn_impl(const char *fn, const psb_index *ix, const float *queries, int64_t q, int32_t k,
                     int32_t *out_ids, float *out_dists, void *stream, int32_t algo, uint32_t variant,
@@ -309,14 +338,32 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
     }
     if (q == 0) return PSB_OK;
     cudaStream_t st = (cudaStream_t)stream;
-    const bool hq = !is_device_ptr(queries);
-    const bool ho = !is_device_ptr(out_ids) || !is_device_ptr(out_dists);
+    // one attribute query per pointer: device memory, or the device address of
+    // page-locked host memory (nullptr for pageable memory)
+    void *mq_dev = nullptr, *mi_dev = nullptr, *md_dev = nullptr;
+    const bool hq = !ptr_info(queries, &mq_dev);
+    const bool hi = !ptr_info(out_ids, &mi_dev), hd = !ptr_info(out_dists, &md_dev);
+    bool hq_mapped = false;
+    const bool ho = hi || hd;
     const float *dq = queries;
     int32_t *di = out_ids;
     float *dd = out_dists;
     cudaError_t e = cudaSuccess;
     const size_t bq = sizeof(float) * (size_t)(q * ix->d), bo = sizeof(float) * (size_t)(q * k);
-    if (hq) {
+    // Pinned host queries are read by the tree kernels in place (zero-copy: each
+    // warp loads its query's d floats once over the host link), so nothing is
+    // staged and no copy precedes the first kernel. They are staged (one copy on
+    // the stream) when many warps read each query: split mode (a query per part)
+    // and brute force (a query per chunk CTA); host-link reads of one address by
+    // thousands of warps cost C3's single-query latency mode 15 us (r02bn).
+    // Pageable queries are always staged.
+    bool staged_q = false;
+    if (hq && mq_dev && parts <= 1 && algo != PSB_ALGO_BRUTE) {
+        dq = static_cast<const float *>(mq_dev);
+        hq_mapped = true;
+    }
+    if (hq && !hq_mapped) {
+        staged_q = true;
         float *tmp = nullptr;
         if ((e = cudaMallocFromPoolAsync((void **)&tmp, bq, ix->pool, st)) != cudaSuccess) return report_cuda(e, fn);
         if ((e = cudaMemcpyAsync(tmp, queries, bq, cudaMemcpyHostToDevice, st)) != cudaSuccess) {
@@ -330,8 +377,8 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
     // the whole result for a copy after the last query; pageable ones are staged.
     bool staged = ho;
     if (ho) {
-        int32_t *mi = is_device_ptr(out_ids) ? out_ids : static_cast<int32_t *>(mapped_host_ptr(out_ids));
-        float *md = is_device_ptr(out_dists) ? out_dists : static_cast<float *>(mapped_host_ptr(out_dists));
+        int32_t *mi = !hi ? out_ids : static_cast<int32_t *>(mi_dev);
+        float *md = !hd ? out_dists : static_cast<float *>(md_dev);
         if (mi && md) {
             di = mi;
             dd = md;
@@ -355,7 +402,7 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
         if (di != out_ids) cudaFreeAsync(di, st);
         if (dd != out_dists) cudaFreeAsync(dd, st);
     }
-    if (hq) cudaFreeAsync((void *)dq, st);
+    if (staged_q) cudaFreeAsync((void *)dq, st);
     return rc;
 }
 

@@ -37,9 +37,15 @@ template <int D, int V>
 int launch_brute_ks(const DevIndex &ix, const float *queries, int64_t nq, int k, int32_t *oi, float *od,
                     cudaStream_t st, int sm, cudaMemPool_t pool);
 
-// Latency-mode helpers (knn_merge.cu): shared pruning distances to +inf, and the
-// filtered merge of [nq][parts][k] per-part lists.
-void init_shared_pd(float *gpd, int64_t nq, cudaStream_t st);
+// Latency-mode helpers (knn_merge.cu): shared pruning distances to +inf (and the
+// task queue, if any, to 0) in one launch, and the filtered merge of [nq][parts][k]
+// per-part lists.
+void init_shared_pd(float *gpd, int64_t nq, unsigned long long *queue, cudaStream_t st);
+
+// cudaOccupancyMaxActiveBlocksPerMultiprocessor, memoised per (kernel, block size,
+// dynamic smem, device): the launchers ask on every call, and a single-query call
+// is latency-bound by host work like this (psb_api.cpp).
+int cached_occupancy(const void *kern, int threads, size_t smem);
 int launch_merge_parts(const int32_t *ids, const float *dists, const float *gpd, int parts, int64_t nq, int k,
                        int32_t *oi, float *od, cudaStream_t st);
 template <int D>
