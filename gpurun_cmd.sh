@@ -1,4 +1,7 @@
-O=gpurun_out/r02bf; mkdir -p $O
-timeout 600 ncu --set full --import-source on --clock-control none -k regex:psb_kernel -s 1 -c 1 -o $O/c5_psb python tools/prof_one.py C5 psb > $O/ncu_c5.log 2>&1
-timeout 600 ncu --set full --import-source on --clock-control none -k regex:bnb_kernel -s 1 -c 1 -o $O/c5_bnb python tools/prof_one.py C5 bnb > $O/ncu_c5b.log 2>&1
-tail -1 $O/ncu_c5.log $O/ncu_c5b.log
+O=gpurun_out/r02bq; mkdir -p $O
+timeout 900 python -m pytest tests -m gpu -x -q > $O/gputests.txt 2>&1
+for r in 1 2; do for c in C2 C5 C3; do
+  PSB_LIB_PATH=$PWD/paper_conf_icpp_namkn16_b200/libpsb_base.so timeout 300 python tools/var_ab.py $c psb 0 > $O/ab_base_${c}_$r.txt 2>&1
+  timeout 300 python tools/var_ab.py $c psb 0 > $O/ab_new_${c}_$r.txt 2>&1
+done; done
+tail -2 $O/gputests.txt; for f in $O/ab_*; do echo "$f $(tail -1 $f | cut -c1-40)"; done

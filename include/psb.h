@@ -172,7 +172,10 @@ int psb_knn_bruteforce(const psb_index *idx, const float *queries, int64_t q, in
  *                          the scan changes the kNN list, Alg. 1 l.41);
  * bit 5 PSB_VAR_PREFETCH_IDS — with every leaf scan, prefetch the leaf's point
  *                          ids into L1 (they are loaded lazily, only for points
- *                          that pass the distance filter).
+ *                          that pass the distance filter). Bits 4 and 5 run the
+ *                          runtime-d kernels (measured slower in batches,
+ *                          DESIGN.md §6; the compile-time-d kernels carry no
+ *                          prefetch code).
  * bit 6 PSB_VAR_P1_INDEX_TIE — pass 1's ClosestLeaf descent (R4) breaks
  *                          MINDIST ties by child index alone. By default a tie
  *                          goes to the child with the smaller MAXDIST first (a
@@ -186,10 +189,9 @@ int psb_knn_bruteforce(const psb_index *idx, const float *queries, int64_t q, in
  *                          smallest MAXDIST over children whose subtrees hold
  *                          >= k points (R3): tighter, and a warp min
  *                          instead of a radix select.
- * bit 8 PSB_VAR_NO_AUTO_PREFETCH — a build with PSB_AUTO_PREFETCH_MIN_D set
- *                          turns bits 4 and 5 on for compile-time d >= that
- *                          value; this bit keeps them off. The default build
- *                          sets no such d (measured slower).
+ * bit 8 PSB_VAR_NO_AUTO_PREFETCH — accepted, no effect: round 1 turned bits 4
+ *                          and 5 on by default at d = 16 and this bit turned them
+ *                          off; no build does so any more.
  * bit 9 PSB_VAR_GENERIC_D — run the runtime-d instantiation of the kernels even
  *                          where a compile-time-d one exists (d, fanout) in
  *                          {(2,32), (3,64), (3,128), (8,128), (16,128)}: the two

@@ -30,15 +30,12 @@ constexpr double REORDER_MIN_BYTES = 64.0 * (1 << 20);
 #define PSB_MINBLOCKS_LARGE_D 6
 #endif
 // PSB prefetched the right sibling's coordinates and the scanned leaf's ids by
-// default at compile-time d >= this in round 1 (C4 16.9 -> 15.9 ms, when the
-// prefetch covered only half of the 8 KB leaf block). Covering the whole block
-// (every line of it) made it a loss: C4 15.3-15.5 ms without it, 16.5-16.7 with
-// both prefetches, 15.6 with the ids alone, 16.3-16.4 with the next leaf alone
-// (profiles/r02_experiments.md). So no d turns it on by default; the variant
-// bits PSB_VAR_PREFETCH_NEXT / _IDS still do.
-#ifndef PSB_AUTO_PREFETCH_MIN_D
-#define PSB_AUTO_PREFETCH_MIN_D 1024   // off: no compile-time d turns the prefetch on
-#endif
+// default at compile-time d = 16 in round 1; covering the whole 8 KB block made it
+// a loss (C4 15.3-15.5 ms without it, 16.5-16.7 with both prefetches,
+// profiles/r02_experiments.md). The variant bits PSB_VAR_PREFETCH_NEXT / _IDS now
+// run the runtime-d kernels, which keep the prefetch code; the compile-time-d
+// kernels carry no prefetch test in their leaf step (2.5 % of the C5 slab's
+// instructions, profiles/r02_experiments.md).
 template <int D>
 struct MinBlocks {
     static constexpr int value = (D == 0 || D >= 16) ? PSB_MINBLOCKS_LARGE_D : PSB_MINBLOCKS_SMALL_D;
@@ -210,8 +207,10 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     int node = 0;
     // Pass-1 state lives in the path cache's unused level-0 slot (no registers
     // held across the loop): p1md[c] = MINDIST of N*'s child c, set to -1 once
-    // that leaf is scanned in pass 1; cache_node[0] = N* (level-1 node id).
+    // that leaf is scanned in pass 1; `nstar` = N* (level-1 node id) once pass 1
+    // is over (-1 before), so pass 2's skip test is one compare in registers.
     float *const p1md = ws.cache_md;
+    int nstar = -1;                                              // N* once pass 1 is over
     int visited = -1;                                            // R10
     while (true) {
         if (lvl > 0) {
@@ -250,7 +249,6 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
                 if (--lvl == 0 && pass1) {                       // ClosestLeaf; keep N*'s MINDISTs
 #pragma unroll
                     for (int t = 0; t < V; ++t) p1md[lane * V + t] = md[t];
-                    if (lane == 0) ws.cache_node[0] = base >> LOGF;
                     __syncwarp();
                 }
             } else {                                             // S7 backtrack (R9)
@@ -264,7 +262,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
             const int j = node;
             bool changed = false;
             // a pass-1 leaf is not scanned again in pass 2 (its points are in the list)
-            const bool pre = !pass1 && (j >> LOGF) == ws.cache_node[0] && p1md[j & (F - 1)] < 0.f;
+            const bool pre = (j >> LOGF) == nstar && p1md[j & (F - 1)] < 0.f;
             if (!pre) changed = scan_leaf<D, V, KS, ST>(ix, j, q, lane, T, k, thr, S, ws.scratch, ws.pf);
             S.step(ws.tr, qi, lane, 0, j, (pass1 ? TR_PASS1 : 0u) | (changed ? TR_CHANGED : 0u) | (pre ? TR_SKIPPED : 0u));
             pd = fminf(pd, key_dist(thr));                       // Alg. 1 l.37
@@ -287,6 +285,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
                     continue;
                 }
                 pass1 = false;                                   // restart at the root
+                nstar = j >> LOGF;
                 lvl = H;
                 node = 0;
                 continue;
@@ -409,7 +408,7 @@ closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, 
 // One warp per query. With `queue` non-null the grid is persistent (as many
 // CTAs as fit on the GPU) and each warp takes the next query from an atomic
 // counter when it finishes one, so a long query never holds an idle block.
-#define PSB_TREE_KERNEL(NAME, BODY, AUTO_PF)                                                         \
+#define PSB_TREE_KERNEL(NAME, BODY)                                                                  \
     template <int D, int V, int KS, bool ST, bool SPH>                                                \
     __global__ void __launch_bounds__(WARPS_PER_CTA * 32, MinBlocks<D>::value)                       \
     NAME(DevIndex ix, const float *__restrict__ queries, int64_t nq, int k,                          \
@@ -421,9 +420,8 @@ closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, 
         const int lane = threadIdx.x & 31;                                                            \
         WarpState ws = warp_state(smem, ix.H, 32 * V, D == 0, KS == 0 ? k : 0);                       \
         ws.tr = tr;                                                                                   \
-        const bool auto_pf = AUTO_PF && D >= PSB_AUTO_PREFETCH_MIN_D && !(variant & PSB_VAR_NO_AUTO_PREFETCH);  \
-        ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) || auto_pf ? PF_NEXT : 0u) |                          \
-                ((variant & PSB_VAR_PREFETCH_IDS) || auto_pf ? PF_IDS : 0u) |                            \
+        ws.pf = ((variant & PSB_VAR_PREFETCH_NEXT) ? PF_NEXT : 0u) |                                   \
+                ((variant & PSB_VAR_PREFETCH_IDS) ? PF_IDS : 0u) |                                     \
                 ((variant & PSB_VAR_P1_INDEX_TIE) ? PF_P1_INDEX_TIE : 0u) |                               \
                 ((variant & PSB_VAR_KTH_MAXDIST) || ix.irregular ? PF_KTH_RULE : 0u);                     \
         const bool use_cache = !(variant & PSB_VAR_NOCACHE);                                          \
@@ -442,8 +440,8 @@ closest_leaf_kernel(DevIndex ix, const float *__restrict__ queries, int64_t nq, 
         }                                                                                             \
     }
 
-PSB_TREE_KERNEL(psb_kernel, psb_query, true)
-PSB_TREE_KERNEL(bnb_kernel, bnb_query, false)
+PSB_TREE_KERNEL(psb_kernel, psb_query)
+PSB_TREE_KERNEL(bnb_kernel, bnb_query)
 
 
 // ---------------------------------------------------------------------------
@@ -902,7 +900,9 @@ int launch_tree_ks(int algo, const DevIndex &ix, const float *queries, int64_t n
                           int32_t *oi, float *od, cudaStream_t st, uint32_t variant, int64_t *stats,
                          cudaMemPool_t pool, int parts, const TraceOut &tr)
 {
-    if (D > 0 && (variant & PSB_VAR_GENERIC_D)) return PSB_NOT_INSTANTIATED;
+    // the prefetch variants run the runtime-d kernels (see PSB_VAR_PREFETCH_* above)
+    if (D > 0 && (variant & (PSB_VAR_GENERIC_D | PSB_VAR_PREFETCH_NEXT | PSB_VAR_PREFETCH_IDS)))
+        return PSB_NOT_INSTANTIATED;
     if (k <= 32) return launch_tree_t<D, V, 1>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts, tr);
     if (k <= 64) return launch_tree_t<D, V, 2>(algo, ix, queries, nq, k, oi, od, st, variant, stats, pool, parts, tr);
     if constexpr (D == 0) {

@@ -677,13 +677,15 @@ __device__ __forceinline__ bool scan_leaf(const DevIndex &ix, int leaf, const Qu
     // next leaf whenever this scan changes the list (Alg. 1 l.41), and this leaf's
     // ids are needed as soon as a distance passes the filter: start both L2->L1
     // transfers now, without holding registers.
-    if ((pf & PF_NEXT) && leaf + 1 < ix.L) {
-        // the whole right-sibling block: d*V lines of 128 B
-        for (int o = lane; o < ix.d * V; o += 32)
-            asm volatile("prefetch.global.L1 [%0];" ::"l"(ix.pts + ((int64_t)leaf + 1) * ix.d * F + o * 32));
+    if constexpr (D == 0) {   // the PSB_VAR_PREFETCH_* variants run the runtime-d kernels only
+        if ((pf & PF_NEXT) && leaf + 1 < ix.L) {
+            // the whole right-sibling block: d*V lines of 128 B
+            for (int o = lane; o < ix.d * V; o += 32)
+                asm volatile("prefetch.global.L1 [%0];" ::"l"(ix.pts + ((int64_t)leaf + 1) * ix.d * F + o * 32));
+        }
+        if ((pf & PF_IDS) && lane < V)
+            asm volatile("prefetch.global.L1 [%0];" ::"l"(ix.ids + (int64_t)leaf * F + lane * 32));
     }
-    if ((pf & PF_IDS) && lane < V)
-        asm volatile("prefetch.global.L1 [%0];" ::"l"(ix.ids + (int64_t)leaf * F + lane * 32));
     constexpr int DC = D;   // compile-time d (0: runtime)
     leaf_dists<D, V>(ix.pts + (int64_t)leaf * (DC > 0 ? DC : ix.d) * F, q, ix.d, lane, dist);
     const float td = key_dist(thr);

@@ -343,6 +343,41 @@ def test_error_codes_on_gpu():
     idx.free()
 
 
+def test_pinned_queries_read_in_place(c2):
+    """Pinned host queries are read by the kernels in place (zero-copy, include/psb.h),
+    also through an interior pointer of a larger pinned tensor, and also by the
+    closest-leaf pre-pass of a reordered batch; split mode and brute force stage them.
+    Every route returns the oracle's rows into pinned and device outputs."""
+    psb = _psb()
+    cfg, pts, qs, idx, exp = c2
+    big = torch.from_numpy(qs[:3000].copy()).pin_memory()
+    sl = slice(517, 2517)                        # interior pointer, 2,000 queries
+    hq = big[sl]
+    e = (exp[0][sl], exp[1][sl])
+    hi = torch.empty((2000, cfg.k), dtype=torch.int32, pin_memory=True)
+    hd = torch.empty((2000, cfg.k), dtype=torch.float32, pin_memory=True)
+    di = torch.empty((2000, cfg.k), dtype=torch.int32, device="cuda")
+    dd = torch.empty((2000, cfg.k), dtype=torch.float32, device="cuda")
+    calls = {
+        "psb": lambda o: psb.psb_knn(idx, hq, cfg.k, out=o),
+        "psb leaf order": lambda o: psb.psb_knn_ex(idx, hq, cfg.k, variant=psb.PSB_VAR_LEAF_ORDER, out=o),
+        "bnb": lambda o: psb.psb_knn_branch_and_bound(idx, hq, cfg.k, out=o),
+        "split 4": lambda o: psb.psb_knn_split(idx, hq, cfg.k, parts=4, out=o),
+        "brute": lambda o: psb.psb_knn_bruteforce(idx, hq, cfg.k, out=o),
+    }
+    for name, call in calls.items():
+        for o in ((hi, hd), (di, dd)):
+            o[0].fill_(-7)
+            ids, d = call(o)
+            torch.cuda.synchronize()
+            assert_same((ids.cpu().numpy(), d.cpu().numpy()), e, f"pinned queries, {name}, out on {o[0].device}")
+    # one query at a time (the latency path): interior pointers of one row
+    for r in (0, 1, 999):
+        ids, d = psb.psb_knn(idx, hq[r:r + 1], cfg.k, out=(hi[:1], hd[:1]))
+        assert np.array_equal(ids.numpy()[0], e[0][r]) and np.array_equal(d.numpy()[0].view(np.uint32),
+                                                                          e[1][r].view(np.uint32))
+
+
 def test_host_buffers_and_stats(c2):
     """Host (pinned and pageable) buffers through the C ABI give identical rows;
     the instrumented entry point changes nothing and its counters are sane."""

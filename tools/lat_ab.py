@@ -24,3 +24,7 @@ print(f"{name} psb: p50/p99 {lat(lambda x: psb.psb_knn(idx, x, cfg.k, out=(hi, h
 for p in map(int, sys.argv[3:]):
     print(f"{name} split parts={p}: p50/p99 {lat(lambda x: psb.psb_knn_split(idx, x, cfg.k, parts=p, out=(hi, hd)))} us",
           flush=True)
+if os.environ.get("LAT_VARIANTS"):
+    for v in map(lambda s: int(s, 0), os.environ["LAT_VARIANTS"].split(",")):
+        print(f"{name} psb variant {v:#x}: p50/p99 "
+              f"{lat(lambda x: psb.psb_knn_ex(idx, x, cfg.k, variant=v, out=(hi, hd)))} us", flush=True)
