@@ -24,9 +24,10 @@
  *  - Queries and outputs may be CUDA device pointers on the index's device or
  *    host memory. Pinned (page-locked, hence device-mapped) host buffers are
  *    used in place by the kernels (zero-copy): result rows are written row by
- *    row as queries finish, and the one-warp-per-query traversals read each
- *    query's d floats over the host link (split mode and brute force, where many
- *    warps read each query, stage pinned queries with one copy). Pageable host
+ *    row as queries finish, and for batches of up to 16,384 queries the
+ *    one-warp-per-query traversals read each query's d floats over the host link
+ *    (larger batches, split mode and brute force, where many warps read each
+ *    query, stage pinned queries with one copy). Pageable host
  *    queries and outputs are staged through stream-ordered device scratch with
  *    cudaMemcpyAsync on `stream`. Either way
  *    the results are in host memory once the stream reaches the end of the call

@@ -312,6 +312,9 @@ static bool ptr_info(const void *p, void **mapped)
     return false;
 }
 
+// Largest batch whose pinned host queries the kernels read in place (knn_impl).
+constexpr int64_t ZERO_COPY_MAX_QUERIES = 16384;
+
 // Launch one algorithm on device buffers. Host buffers: pinned ones are used in
 // place by the kernels (zero-copy queries and result rows), pageable ones are
 // staged through stream-ordered device scratch with copies on the same stream.
@@ -350,15 +353,18 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
     float *dd = out_dists;
     cudaError_t e = cudaSuccess;
     const size_t bq = sizeof(float) * (size_t)(q * ix->d), bo = sizeof(float) * (size_t)(q * k);
-    // Pinned host queries are read by the tree kernels in place (zero-copy: each
-    // warp loads its query's d floats once over the host link), so nothing is
-    // staged and no copy precedes the first kernel. They are staged (one copy on
-    // the stream) when many warps read each query: split mode (a query per part)
-    // and brute force (a query per chunk CTA); host-link reads of one address by
-    // thousands of warps cost C3's single-query latency mode 15 us (r02bn).
-    // Pageable queries are always staged.
+    // Pinned host queries of a small batch are read by the tree kernels in place
+    // (zero-copy: each warp loads its query's d floats over the host link), so
+    // nothing is staged and no copy precedes the first kernel: C2's e2e
+    // 47.7 -> 50.5 M q/s, single-query p50 -10 us. They are staged (one bulk copy
+    // on the stream) when many warps read each query (split mode: a query per
+    // part; brute force: a query per chunk CTA; host-link reads of one address by
+    // thousands of warps cost C3's latency mode 15 us, r02bn) and for large
+    // batches, where 10^6 small host-link reads (the closest-leaf pre-pass and the
+    // traversal each read every query) cost more than one copy (C5 slab e2e
+    // 97.8 -> 92.4 M q/s, r02bv). Pageable queries are always staged.
     bool staged_q = false;
-    if (hq && mq_dev && parts <= 1 && algo != PSB_ALGO_BRUTE) {
+    if (hq && mq_dev && parts <= 1 && algo != PSB_ALGO_BRUTE && q <= ZERO_COPY_MAX_QUERIES) {
         dq = static_cast<const float *>(mq_dev);
         hq_mapped = true;
     }

@@ -371,6 +371,12 @@ def test_pinned_queries_read_in_place(c2):
             ids, d = call(o)
             torch.cuda.synchronize()
             assert_same((ids.cpu().numpy(), d.cpu().numpy()), e, f"pinned queries, {name}, out on {o[0].device}")
+    # a batch above the zero-copy limit (16,384 queries): staged with one copy
+    big2 = torch.from_numpy(np.concatenate([qs, qs])).pin_memory()
+    ids, d = psb.psb_knn(idx, big2, cfg.k)
+    torch.cuda.synchronize()
+    assert_same((ids.numpy(), d.numpy()), (np.concatenate([exp[0], exp[0]]), np.concatenate([exp[1], exp[1]])),
+                "pinned queries above the zero-copy limit")
     # one query at a time (the latency path): interior pointers of one row
     for r in (0, 1, 999):
         ids, d = psb.psb_knn(idx, hq[r:r + 1], cfg.k, out=(hi[:1], hd[:1]))
