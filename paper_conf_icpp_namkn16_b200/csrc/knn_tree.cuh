@@ -611,6 +611,7 @@ __device__ __forceinline__ void psb_node_query(const DevIndex &ix, const float *
     Stats<ST> S;
     float *const p1md = ws.cache_md;                             // N*'s child MINDISTs (pass 1)
     bool pass1 = true;
+    int nstar = -1;                                              // N* once pass 1 is over
     int lvl = H, node = 0, visited = -1;
     while (true) {
         if (lvl > 0) {
@@ -671,7 +672,6 @@ __device__ __forceinline__ void psb_node_query(const DevIndex &ix, const float *
                 if (--lvl == 0 && pass1) {
 #pragma unroll
                     for (int t = 0; t < V; ++t) p1md[lane * V + t] = md[t];
-                    if (lane == 0) ws.cache_node[0] = base >> LOGF;
                     __syncwarp();
                 }
             } else {                                             // S7 backtrack (R9)
@@ -683,7 +683,7 @@ __device__ __forceinline__ void psb_node_query(const DevIndex &ix, const float *
         } else {
             const int j = node;
             bool changed = false;
-            const bool pre = !pass1 && (j >> LOGF) == ws.cache_node[0] && p1md[j & (F - 1)] < 0.f;
+            const bool pre = (j >> LOGF) == nstar && p1md[j & (F - 1)] < 0.f;
             if (!pre) changed = scan_leaf<D, V, KS, ST>(ix, j, q, lane, T, k, thr, S, ws.scratch, ws.pf);
             pd = fminf(pd, key_dist(thr));
             if (pd < published) {
@@ -709,6 +709,7 @@ __device__ __forceinline__ void psb_node_query(const DevIndex &ix, const float *
                     continue;
                 }
                 pass1 = false;
+                nstar = j >> LOGF;
                 lvl = H;
                 node = 0;
                 continue;
