@@ -471,7 +471,7 @@ int psb_knn_split(const psb_index *ix, const float *queries, int64_t q, int32_t 
             }
         } else if (q < 4 * resident) {
             if (work >= 64.0) {
-                p = 12 * resident / q;
+                p = 14 * resident / q;             // C4: 6 parts (8.11 ms; 5: 8.33, 7: 8.13, 8: 8.45; r02by)
                 p = p < 2 ? 2 : (p > 8 ? 8 : p);
             }
         }
