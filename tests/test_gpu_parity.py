@@ -206,6 +206,23 @@ def test_c5_slab_full_batch_sampled():
     idx.free()
 
 
+def test_ctx_paper_shape_all_rows():
+    """SURVEY §8(d) "ctx": the paper's experiment shape (64-D clustered, n=10^6,
+    F=128, 240 queries, k=32; runtime-d kernels), every row of PSB, PSB latency
+    mode, B&B and brute force against the oracle's brute force."""
+    psb = _psb()
+    cfg = W.config("CTX")
+    pts, qs = cfg.points(), cfg.queries()
+    idx = psb.psb_build(pts, cfg.fanout)
+    exp = oracle.knn_bruteforce(pts, qs, cfg.k)
+    for algo in ("psb", "bnb", "brute"):
+        assert_same(run(idx, qs, cfg.k, algo), exp, f"CTX {algo}")
+    si, sd = psb.psb_knn_split(idx, torch.from_numpy(qs).cuda(), cfg.k, parts=0)
+    torch.cuda.synchronize()
+    assert_same((si.cpu().numpy(), sd.cpu().numpy()), exp, "CTX psb split (auto)")
+    idx.free()
+
+
 @pytest.mark.parametrize("case", [
     dict(n=1, d=2, F=32, k=4), dict(n=31, d=3, F=32, k=40), dict(n=33, d=3, F=32, k=33),
     dict(n=1000, d=1, F=32, k=10), dict(n=5000, d=5, F=64, k=20), dict(n=3000, d=64, F=32, k=9),

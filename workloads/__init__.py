@@ -160,6 +160,9 @@ CONFIGS = {
     "C3": Config("C3", "uniform", 4_000_000, 8, 128, 100_000, 16, cfg_id=3),
     "C4": Config("C4", "clustered", 16_000_000, 16, 128, 10_000, 64, cfg_id=4),
     "C5": Config("C5", "uniform", 512_000_000, 3, 128, 1_000_000, 32, cfg_id=5),
+    # SURVEY.md §8(d) "ctx": the paper's own experiment shape (§V-B: 64-D
+    # clustered points, 240 kNN queries), optional context, not a BASELINE config
+    "CTX": Config("CTX", "clustered", 1_000_000, 64, 128, 240, 32, cfg_id=6),
 }
 
 
