@@ -298,8 +298,10 @@ static bool is_device_ptr(const void *p)
 }
 
 // true for device (or managed) memory; otherwise *mapped = the device address of
-// page-locked (pinned or registered) host memory, nullptr for pageable memory.
-static bool ptr_info(const void *p, void **mapped)
+// page-locked (pinned or registered) host memory registered by device `dev`'s
+// context, nullptr for pageable memory (or memory pinned by another device's
+// context, which is then staged like pageable memory).
+static bool ptr_info(const void *p, int dev, void **mapped)
 {
     *mapped = nullptr;
     cudaPointerAttributes a;
@@ -308,7 +310,7 @@ static bool ptr_info(const void *p, void **mapped)
         return false;
     }
     if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) return true;
-    if (a.type == cudaMemoryTypeHost) *mapped = a.devicePointer;
+    if (a.type == cudaMemoryTypeHost && a.device == dev) *mapped = a.devicePointer;
     return false;
 }
 
@@ -344,8 +346,8 @@ static int knn_impl(const char *fn, const psb_index *ix, const float *queries, i
     // one attribute query per pointer: device memory, or the device address of
     // page-locked host memory (nullptr for pageable memory)
     void *mq_dev = nullptr, *mi_dev = nullptr, *md_dev = nullptr;
-    const bool hq = !ptr_info(queries, &mq_dev);
-    const bool hi = !ptr_info(out_ids, &mi_dev), hd = !ptr_info(out_dists, &md_dev);
+    const bool hq = !ptr_info(queries, ix->device, &mq_dev);
+    const bool hi = !ptr_info(out_ids, ix->device, &mi_dev), hd = !ptr_info(out_dists, ix->device, &md_dev);
     bool hq_mapped = false;
     const bool ho = hi || hd;
     const float *dq = queries;
