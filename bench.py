@@ -494,7 +494,8 @@ def main():
             dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
         extras["e2e"] = {"value": units * args.steps / (float(e2e_t.item()) / 1e3), "unit": UNIT,
                          "h2d_bytes_per_step": int(ql * idx.d * 4), "d2h_bytes_per_step": int(ql * k * 8),
-                         "api": "psb_knn_ex with pinned host buffers (library copies the queries H2D on the stream; "
+                         "api": "psb_knn_ex with pinned host buffers (batches of <= 16,384 queries: the kernels read "
+                                "the queries in place over the host link; larger batches: one H2D copy on the stream; "
                                 "the kernel writes each result row straight into the pinned host output)"}
         if args.mode == "data" and world > 1:
             extras["e2e"]["note"] = "local search only (the data-sharded exchange runs on device buffers)"
