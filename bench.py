@@ -280,12 +280,12 @@ def roofline(algo, idx, q, k, alg_bytes, kern_s, prof_cfg, l2_peak):
         prim = {"bound": "l2", "achieved": a, "peak": l2_peak, "unit": "GB/s", "frac": a / l2_peak,
                 "l2_bytes_per_launch": l2b, "note": "split mode has no per-part traversal counters: "
                 "achieved = ncu lts bytes of psb_split_kernel (profiles/traffic.json) / live launch time",
-                "peak_source": "measured in this run: psb_probe_l2_read (64 MiB L2-resident, ld.global.cg)"}
+                "peak_source": "measured in this run: psb_probe_l2_read (64 MiB L2-resident; best of 16-B x1, 16-B x4, 32-B x1, 32-B x2 ld.global.cg loads per thread)"}
     else:
         a = alg_bytes / kern_s / 1e9
         prim = {"bound": "l2", "achieved": a, "peak": l2_peak, "unit": "GB/s", "frac": a / l2_peak,
                 "algorithmic_bytes_per_launch": alg_bytes,
-                "peak_source": "measured in this run: psb_probe_l2_read (64 MiB L2-resident, ld.global.cg)"}
+                "peak_source": "measured in this run: psb_probe_l2_read (64 MiB L2-resident; best of 16-B x1, 16-B x4, 32-B x1, 32-B x2 ld.global.cg loads per thread)"}
     dram = traffic_from_profiles(prof_cfg, algo, "dram_bytes_per_launch")
     prim["traffic"] = dram
     prim["avg_launch_ms"] = kern_s * 1e3

@@ -361,8 +361,10 @@ int psb_build_host_blob(const float *points, int64_t n, int32_t d, int32_t fanou
  * the traversal's node and leaf blocks are served mostly from L2, so that is the
  * memory ceiling their algorithmic bytes are compared with). A `bytes` buffer
  * (>= 1 MiB; 64 MiB fits B200's L2) is read once to make it L2-resident, then
- * `passes` times per timed launch with 16-byte L2-only (ld.global.cg) loads by
- * 4 x 512 threads per SM; *gbs = the best of `reps` CUDA-event-timed launches.
+ * `passes` times per timed launch with L2-only (ld.global.cg) loads by 4 x 512
+ * threads per SM, in four shapes (one or four 16-byte loads in flight per thread,
+ * one or two 32-byte loads); *gbs = the best of `reps` CUDA-event-timed launches
+ * over all shapes (one 16-byte load per thread under-reads the L2 by ~20 %).
  * Synchronous; allocates and frees its own buffer. */
 int psb_probe_l2_read(int64_t bytes, int32_t passes, int32_t reps, double *gbs);
 
