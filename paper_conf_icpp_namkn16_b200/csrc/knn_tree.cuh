@@ -214,19 +214,17 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     int visited = -1;                                            // R10
     // Pass 2's eligibility at the current level-1 node (the node every non-changing
     // leaf returns to, Alg. 1 l.44): this lane's bits of {c < c_end : MINDIST <= pd}
-    // for node enode, computed at pruning distance epd. While the walk returns to
-    // the same node with the same pd, the set is the same (the node is in the path
-    // cache, MINDIST is a pure function of (query, node)), so the next child is the
-    // next bit above `visited` without re-reading or re-testing the MINDISTs.
-    // Compiled in where it pays: d >= 8 (C3 5.57 -> 5.13 ms, C4 14.75 -> 13.8 ms);
-    // at d = 3 most returns follow a change of pd, and the test itself costs (C5
-    // slab 9.75 -> 9.98 ms, C2 +1 %; profiles/r02ci).
+    // for node enode. While the walk returns to the same node and pd has not moved,
+    // the set is the same (the node is in the path cache, MINDIST is a pure function
+    // of (query, node)), so the next child is the next bit above `visited` without
+    // re-reading or re-testing the MINDISTs.
+    // The set stays valid until pd can change: a leaf scan that changed the list, or
+    // a node fetch (its MAXDIST bound); both reset enode.
     constexpr bool REUSE_L1 = D == 0 || D >= 8;
     unsigned emask = 0;
     int enode = -1;
-    float epd = 0.f;
     while (true) {
-        if (REUSE_L1 && lvl == 1 && node == enode && pd == epd && use_cache) {
+        if (REUSE_L1 && lvl == 1 && node == enode && use_cache) {
             // same walk as the generic step below on a path-cache hit
             S.node(false);
             S.step(ws.tr, qi, lane, 1, node, 0u);
@@ -249,6 +247,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
         if (lvl > 0) {
             float md[V], Md[V];
             const bool fetched = internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md, Md);
+            if (REUSE_L1 && fetched) enode = -1;                 // pd may have fallen
             S.node(fetched);
             S.step(ws.tr, qi, lane, lvl, node, (pass1 ? TR_PASS1 : 0u) | (fetched ? TR_FETCHED : 0u));
             const int base = node * F;
@@ -271,7 +270,6 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
                 if (REUSE_L1 && lvl == 1) {                      // remembered for the next returns
                     emask = under;
                     enode = node;
-                    epd = pd;
                 }
                 const unsigned mine = under & ~((1u << lo_b) - 1u);
                 const unsigned bal = __ballot_sync(FULL, mine != 0);
@@ -302,6 +300,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
             // a pass-1 leaf is not scanned again in pass 2 (its points are in the list)
             const bool pre = (j >> LOGF) == nstar && p1md[j & (F - 1)] < 0.f;
             if (!pre) changed = scan_leaf<D, V, KS, ST>(ix, j, q, lane, T, k, thr, S, ws.scratch, ws.pf);
+            if (REUSE_L1 && changed) enode = -1;                 // pd may have fallen
             S.step(ws.tr, qi, lane, 0, j, (pass1 ? TR_PASS1 : 0u) | (changed ? TR_CHANGED : 0u) | (pre ? TR_SKIPPED : 0u));
             pd = fminf(pd, key_dist(thr));                       // Alg. 1 l.37
             if (pass1) {
