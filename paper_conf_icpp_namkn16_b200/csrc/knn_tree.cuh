@@ -36,6 +36,9 @@ constexpr double REORDER_MIN_BYTES = 64.0 * (1 << 20);
 // run the runtime-d kernels, which keep the prefetch code; the compile-time-d
 // kernels carry no prefetch test in their leaf step (2.5 % of the C5 slab's
 // instructions, profiles/r02_experiments.md).
+#ifndef PSB_REUSE_L1_MIN_D
+#define PSB_REUSE_L1_MIN_D 8   // eligibility reuse in pass 2 for compile-time d >= this (psb_query)
+#endif
 template <int D>
 struct MinBlocks {
     static constexpr int value = (D == 0 || D >= 16) ? PSB_MINBLOCKS_LARGE_D : PSB_MINBLOCKS_SMALL_D;
@@ -220,7 +223,7 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     // re-reading or re-testing the MINDISTs.
     // The set stays valid until pd can change: a leaf scan that changed the list, or
     // a node fetch (its MAXDIST bound); both reset enode.
-    constexpr bool REUSE_L1 = D == 0 || D >= 8;
+    constexpr bool REUSE_L1 = D == 0 || D >= PSB_REUSE_L1_MIN_D;
     unsigned emask = 0;
     int enode = -1;
     while (true) {
