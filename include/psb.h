@@ -167,8 +167,11 @@ int psb_knn_bruteforce(const psb_index *idx, const float *queries, int64_t q, in
  *                          the leaf PSB's pass 1 descends to (Alg. 1 l.3),
  *                          so warps running together walk neighbouring leaves and
  *                          share them in L1/L2. Rows are still written in input
- *                          order. With neither bit, leaf order is used when
- *                          q >= 1024 and the leaves (points + ids) exceed 64 MiB.
+ *                          order. With neither bit, the batch is ordered when
+ *                          q >= 1024 and the leaves (points + ids) exceed 64 MiB:
+ *                          by ClosestLeaf for d > 4, by the queries' Hilbert key
+ *                          over the data's bounding box for d <= 4 (no node reads;
+ *                          C5 slab 9.74 -> 9.24 ms).
  * bit 4 PSB_VAR_PREFETCH_NEXT — with every leaf scan, prefetch the right
  *                          sibling's coordinates into L1 (the next leaf whenever
  *                          the scan changes the kNN list, Alg. 1 l.41);

@@ -73,6 +73,7 @@ struct psb_index {
     float *pts = nullptr;
     int32_t *ids = nullptr;
     float *nodes = nullptr;
+    float *box = nullptr;           // bounding box of the real points [2][d] (batch ordering)
     int64_t device_bytes = 0;
     int32_t sphere = 0, blk_floats = 0;
     int32_t irregular = 0;          // imported with non-full leaves (DevIndex::irregular)
@@ -88,6 +89,7 @@ static void index_release(psb_index *ix)
     cudaFree(ix->pts);
     cudaFree(ix->ids);
     cudaFree(ix->nodes);
+    cudaFree(ix->box);
     if (ix->pool) cudaMemPoolDestroy(ix->pool);
     if (prev >= 0) cudaSetDevice(prev);
     delete ix;
@@ -100,6 +102,7 @@ static DevIndex dev_view(const psb_index *ix)
     v.pts = ix->pts;
     v.ids = ix->ids;
     v.nodes = ix->nodes;
+    v.box = ix->box;
     for (int l = 0; l <= PSB_MAXLVL; ++l) {
         v.level_off[l] = ix->level_off[l];
         v.nlev[l] = ix->nlev[l];
@@ -138,6 +141,17 @@ static int make_pool(psb_index *ix, const char *fn)
     uint64_t keep = UINT64_MAX;
     cudaMemPoolSetAttribute(ix->pool, cudaMemPoolAttrReleaseThreshold, &keep);
     return PSB_OK;
+}
+
+// The bounding box of the index's points (the Hilbert batch order, knn_order.cu).
+static int attach_box(psb_index *ix, const char *fn)
+{
+    cudaError_t e = cudaMalloc((void **)&ix->box, sizeof(float) * 2 * (size_t)ix->d);
+    if (e != cudaSuccess) return report_cuda(e, fn);
+    int rc = psb::index_box(ix->pts, ix->ids, ix->L, ix->d, ix->F, ix->box, 0);
+    if (rc == PSB_OK) rc = report_cuda(cudaStreamSynchronize(0), fn);
+    ix->device_bytes += (int64_t)(sizeof(float) * 2 * ix->d);
+    return rc;
 }
 
 extern "C" {
@@ -252,7 +266,7 @@ int psb_build_ex(const float *points, int64_t n, int32_t d, int32_t fanout, int6
         }
     }
     ix->device_bytes = (int64_t)(bp + bi + bn);
-    if ((rc = make_pool(ix, "psb_build_ex")) != PSB_OK) {
+    if ((rc = attach_box(ix, "psb_build_ex: bounding box")) != PSB_OK || (rc = make_pool(ix, "psb_build_ex")) != PSB_OK) {
         index_release(ix);
         return rc;
     }
@@ -693,7 +707,8 @@ int psb_index_import(const void *blob, int64_t size, psb_index **out)
         return rc;
     }
     ix->device_bytes = (int64_t)(bp + bi + bn);
-    if ((rc = make_pool(ix, "psb_index_import")) != PSB_OK) {
+    if ((rc = attach_box(ix, "psb_index_import: bounding box")) != PSB_OK ||
+        (rc = make_pool(ix, "psb_index_import")) != PSB_OK) {
         index_release(ix);
         return rc;
     }

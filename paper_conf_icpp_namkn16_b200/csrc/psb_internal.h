@@ -6,6 +6,11 @@
 #include "psb.h"
 
 #define PSB_MAXLVL 8   // internal levels; F=32 and n < 2^31 need at most 6
+// Large batches at d <= this are ordered by Hilbert key instead of closest leaf
+// (knn_order.cu; DESIGN.md §6 "Batch scheduling").
+#ifndef PSB_HILBERT_ORDER_MAX_D
+#define PSB_HILBERT_ORDER_MAX_D 4
+#endif
 
 // Flat index as laid out in HBM (DESIGN.md §4 "Data layout in HBM").
 //   pts   [L][d][F]  leaf-blocked SoA point coordinates (pad slots +inf)
@@ -19,6 +24,7 @@ struct DevIndex {
     const float *pts;
     const int32_t *ids;
     const float *nodes;
+    const float *box;                   // bounding box of the real points [2][d] (lo, hi)
     int64_t level_off[PSB_MAXLVL + 1];  // float offset of level l's first block (l >= 1)
     int64_t nlev[PSB_MAXLVL + 1];       // nodes per level, nlev[0] = L
     int64_t span[PSB_MAXLVL + 1];       // leaves per full subtree at level l (clamped)

@@ -57,6 +57,13 @@ int launch_brute_v(const DevIndex &ix, const float *queries, int64_t nq, int k, 
 int gpu_bulk_load(const float *d_points, const GpuLayoutShape &sh, int64_t id_base, float *pts, int32_t *ids,
                   float *nodes, cudaStream_t st, bool sphere, int kmeans_iters);
 
+// Batch order by Hilbert key for d <= PSB_HILBERT_ORDER_MAX_D (knn_order.cu):
+// order[i] = the input row processed i-th, keys over the index box (index_box).
+int hilbert_query_order(const float *queries, int64_t nq, int d, const float *box, int32_t *order, cudaMemPool_t pool,
+                        cudaStream_t st);
+// Bounding box of an index's real points into box[2d] (lo row, hi row). Async.
+int index_box(const float *pts, const int32_t *ids, int64_t L, int d, int F, float *box, cudaStream_t st);
+
 // Stable sort of queries by closest-leaf id (knn_order.cu): order[i] = the input
 // row processed i-th. leaf_key is [nq] device memory; order is [nq].
 int sort_query_order(const uint32_t *leaf_key, int64_t nq, int64_t L, int32_t *order, cudaMemPool_t pool,
