@@ -310,18 +310,21 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
                 const int b1 = j & ~(F - 1);                     // N*'s first leaf
                 if (lane == 0) p1md[j - b1] = -1.f;              // scanned
                 __syncwarp();
-                // next leaf of N* in (MINDIST, index) order, if its MINDIST <= pd
-                u64 best = ~0ull;
+                // next leaf of N* in (MINDIST, index) order, if its MINDIST <= pd:
+                // the smallest MINDIST bit pattern (non-negative floats order like
+                // their bits) by one REDUX, then the smallest index holding it
+                uint32_t mb = 0xffffffffu, mc = 0xffffffffu;
 #pragma unroll
                 for (int t = 0; t < V; ++t) {
                     const int cc = lane * V + t;
                     const float v = p1md[cc];
-                    const u64 kk = make_key(v, cc);
-                    if (v >= 0.f && b1 + cc < (int)ix.L && kk < best) best = kk;
+                    const uint32_t bits = (v >= 0.f && b1 + cc < (int)ix.L) ? __float_as_uint(v) : 0xffffffffu;
+                    if (bits < mb) { mb = bits; mc = (uint32_t)cc; }
                 }
-                best = warp_min_u64(best);
-                if (best != ~0ull && key_dist(best) <= pd) {
-                    node = b1 + (int)(best & 0xffffffffu);
+                const uint32_t gm = __reduce_min_sync(FULL, mb);
+                const uint32_t gc = __reduce_min_sync(FULL, mb == gm ? mc : 0xffffffffu);
+                if (gm != 0xffffffffu && __uint_as_float(gm) <= pd) {
+                    node = b1 + (int)gc;
                     continue;
                 }
                 pass1 = false;                                   // restart at the root
