@@ -1,6 +1,6 @@
-O=gpurun_out/r02bw; mkdir -p $O
-timeout 900 python -m pytest tests -m gpu -x -q > $O/gputests.txt 2>&1
-timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.txt 2>&1
-timeout 600 python bench.py --config C2 > $O/bench_C2.json 2> $O/bench_C2.err
-timeout 900 python bench.py --config C5 --mode data --slab 8 --steps 50 > $O/bench_C5slab.json 2> $O/bench_C5slab.err
-tail -2 $O/gputests.txt; cat $O/smoke.txt
+O=gpurun_out/r02db; mkdir -p $O
+for r in 1 2; do for c in C3 C4 C5; do
+  timeout 300 python tools/var_ab.py $c psb 0 > $O/ab_base_${c}_$r.txt 2>&1
+  for v in 0 50; do PSB_LIB_PATH=$PWD/paper_conf_icpp_namkn16_b200/libpsb_co$v.so timeout 300 python tools/var_ab.py $c psb 0 > $O/ab_co${v}_${c}_$r.txt 2>&1; done
+done; done
+for f in $O/ab_*; do echo "$f $(tail -1 $f | cut -c1-40)"; done
