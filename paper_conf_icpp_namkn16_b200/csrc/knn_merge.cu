@@ -38,9 +38,13 @@ merge_kernel(const int32_t *__restrict__ ids, const float *__restrict__ dists, i
     T.store(k, lane, out_ids + qi * k, out_dists + qi * k);
 }
 
-// Latency-mode merge: one CTA of MP_WARPS warps per query; warp w takes parts
-// w, w+MP_WARPS, ...; only keys with dist <= the query's final shared pruning
-// distance can belong to the answer, so the rest are dropped before any id load.
+// Latency-mode merge: one CTA of MP_WARPS warps per query. Only keys with dist <=
+// the query's final shared pruning distance can belong to the answer (every true
+// neighbour is, and few others are), so the whole [parts][k] block is first read
+// at once by all threads (one L2 round trip) and the survivors are collected in
+// shared memory (the per-warp lists' space); one warp then keeps the k smallest.
+// If more keys survive than that space holds (ties at the bound), the per-warp
+// merge below runs instead.
 constexpr int MP_WARPS = 32;
 
 template <int KS>
@@ -50,12 +54,42 @@ merge_parts_kernel(const int32_t *__restrict__ ids, const float *__restrict__ di
 {
     __shared__ u64 lists[MP_WARPS][KS * 32];
     __shared__ u64 scratch_all[MP_WARPS][32];
+    __shared__ int nbuf;
+    constexpr int MP_BUF = MP_WARPS * KS * 32;
+    u64 *const buf = &lists[0][0];                   // the fast path's survivors
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t qi = blockIdx.x;
     const float lim = __ldg(gpd + qi);
     TopK<KS> T;
     T.init();
     u64 thr = PAD_KEY;
+    if (threadIdx.x == 0) nbuf = 0;
+    __syncthreads();
+    {
+        const int total = parts * k;
+        const float *dq = dists + qi * (int64_t)total;
+        const int32_t *iq = ids + qi * (int64_t)total;
+#pragma unroll 8
+        for (int i = threadIdx.x; i < total; i += MP_WARPS * 32) {
+            const float dv = __ldg(dq + i);
+            if (dv <= lim) {
+                const int pos = atomicAdd(&nbuf, 1);
+                if (pos < MP_BUF) buf[pos] = make_key(dv, __ldg(iq + i));
+            }
+        }
+    }
+    __syncthreads();
+    const int nb = nbuf;
+    if (nb <= MP_BUF) {
+        if (w == 0) {
+            for (int c = 0; c < nb; c += 32) {
+                u64 cand[1] = {c + lane < nb ? buf[c + lane] : ~0ull};
+                T.template offer<1>(cand, k, lane, thr, scratch_all[0]);
+            }
+            T.store(k, lane, out_ids + qi * k, out_dists + qi * k);
+        }
+        return;
+    }
     constexpr int U = 4;
     for (int p0 = w; p0 < parts; p0 += MP_WARPS * U) {
         float dv[U][KS];
