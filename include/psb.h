@@ -133,7 +133,7 @@ int psb_knn(const psb_index *idx, const float *queries, int64_t q, int32_t k,
  *    so the eligible leaves of a query, which cluster in neighbouring nodes, are
  *    spread over all parts: this shortens the long queries that end a batch.
  * parts = 0 picks, with W = (1 + (min(k,F)/F)^(1/d))^d the classic uniform-data
- * estimate of the leaves a query touches: ~16 warps per SM in total (at least 32
+ * estimate of the leaves a query touches: ~16 warps per SM in total (at least 16
  * leaves per part) for q <= 8 x SMs when W >= 16; 2-8 parts (14 x resident warps / q)
  * for batches of fewer
  * than 128 x SMs queries when W >= 64; else 1.

@@ -468,7 +468,7 @@ int psb_knn_split(const psb_index *ix, const float *queries, int64_t q, int32_t 
     if (ix && parts == 0) {
         // auto (DESIGN.md §6 "split mode"):
         //  - few queries (<= 1/4 of the resident warps): latency mode, about 16
-        //    warps per SM in total, at least 32 leaves per part, when the
+        //    warps per SM in total, at least 16 leaves per part, when the
         //    estimated leaves per query (below) reach 16;
         //  - a batch that fills the GPU less than 4 times over, of queries that
         //    touch many leaves: 2-8 parts per query against the batch's tail. The
@@ -482,7 +482,7 @@ int psb_knn_split(const psb_index *ix, const float *queries, int64_t q, int32_t 
         if (q * 4 <= resident) {
             if (work >= 16.0) {                   // else one warp is faster than the split's overhead
                 p = q > 0 ? (int64_t)ix->sm_count * 16 / q : 1;
-                const int64_t pmax = ix->L / 32;     // C3: 976 parts, p50 83.5 us (1,953: 93.5; r02bz)
+                const int64_t pmax = ix->L / 16;     // C3: 1,953 parts, p50 72 us (976: 79; r02de)
                 if (p > pmax) p = pmax;
             }
         } else if (q < 4 * resident) {
