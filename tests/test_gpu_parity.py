@@ -206,6 +206,28 @@ def test_c5_slab_full_batch_sampled():
     idx.free()
 
 
+@pytest.mark.parametrize("d,n", [(2, 9_000_000), (4, 4_000_000)])
+def test_hilbert_batch_order_low_d(d, n):
+    """Large batches at d <= 4 are ordered by the queries' Hilbert key (knn_order.cu):
+    leaves above 64 MiB and >= 1,024 queries, so the d = 2 (16 bits per axis) and
+    d = 4 (8 bits) key paths run; rows equal to the oracle, and to the closest-leaf
+    order (PSB_VAR_LEAF_ORDER) and the input order, for PSB and B&B."""
+    psb = _psb()
+    pts = W.gen_uniform(n, d, 0xB0 + d)
+    qs = W.gen_uniform(4000, d, 0xB1 + d)
+    qs[:50] = qs[:50] * 3.0 - 1.0                     # some queries outside the data's box
+    idx = psb.psb_build(pts, 64)
+    sub = np.arange(0, 4000, 20)
+    exp = oracle.knn_bruteforce(pts, qs[sub], 16)
+    for algo in ("psb", "bnb"):
+        got = run(idx, qs, 16, algo)
+        assert_same((got[0][sub], got[1][sub]), exp, f"d={d} {algo} Hilbert order")
+        for var in (psb.PSB_VAR_LEAF_ORDER, psb.PSB_VAR_INPUT_ORDER):
+            other = run(idx, qs, 16, algo, var)
+            assert np.array_equal(other[0], got[0]) and np.array_equal(other[1].view(np.uint32), got[1].view(np.uint32))
+    idx.free()
+
+
 def test_ctx_paper_shape_all_rows():
     """SURVEY §8(d) "ctx": the paper's experiment shape (64-D clustered, n=10^6,
     F=128, 240 queries, k=32; runtime-d kernels), every row of PSB, PSB latency
