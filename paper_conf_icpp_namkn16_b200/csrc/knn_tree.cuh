@@ -227,26 +227,6 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
     unsigned emask = 0;
     int enode = -1;
     while (true) {
-        if (REUSE_L1 && lvl == 1 && node == enode && use_cache) {
-            // same walk as the generic step below on a path-cache hit
-            S.node(false);
-            S.step(ws.tr, qi, lane, 1, node, 0u);
-            const int base = node * F;
-            const int lo_b = min(max(visited + 1 - base - lane * V, 0), V);
-            const unsigned mine = emask & ~((1u << lo_b) - 1u);
-            const unsigned bal = __ballot_sync(FULL, mine != 0);
-            if (bal) {                                           // leftmost (R6, R7)
-                const int src = __ffs(bal) - 1;
-                node = base + src * V + (__ffs(__shfl_sync(FULL, mine, src)) - 1);
-                lvl = 0;
-            } else {                                             // S7 backtrack (R9)
-                if (lvl == H) break;                             // root exhausted (R10)
-                visited = max_leaf(ix, 1, node);
-                node /= F;
-                lvl = 2;
-            }
-            continue;
-        }
         if (lvl > 0) {
             float md[V], Md[V];
             const bool fetched = internal_md<D, V, SPH>(ix, lvl, node, q, lane, ws, use_cache, use_max, k, pd, md, Md);
@@ -340,6 +320,26 @@ __device__ __forceinline__ void psb_query(const DevIndex &ix, const float *__res
             } else {
                 node = j / F;                                    // l.44 parent link
                 lvl = 1;
+                if (REUSE_L1 && node == enode && use_cache) {
+                    // the parent's visit without leaving the leaf step: the same
+                    // walk as the generic step on a path-cache hit
+                    S.node(false);
+                    S.step(ws.tr, qi, lane, 1, node, 0u);
+                    const int base = node * F;
+                    const int lo_b = min(max(j + 1 - base - lane * V, 0), V);
+                    const unsigned mine = emask & ~((1u << lo_b) - 1u);
+                    const unsigned bal = __ballot_sync(FULL, mine != 0);
+                    if (bal) {                                   // leftmost (R6, R7)
+                        const int src = __ffs(bal) - 1;
+                        node = base + src * V + (__ffs(__shfl_sync(FULL, mine, src)) - 1);
+                        lvl = 0;
+                    } else {                                     // S7 backtrack (R9)
+                        if (H == 1) break;                       // root exhausted (R10)
+                        visited = max_leaf(ix, 1, node);
+                        node /= F;
+                        lvl = 2;
+                    }
+                }
             }
         }
     }
