@@ -665,11 +665,18 @@ __device__ __forceinline__ void psb_node_query(const DevIndex &ix, const float *
             const int base = node * F;
             const int c_end = min(F, (int)ix.nlev[lvl - 1] - base);
             // this lane's children lane*V+t that exist and, at level 2, are owned
+            // (child ids base+lane*V+t are consecutive: one modulo per lane)
             unsigned mine = 0;
+            if (lvl == 2) {
+                int r = (base + lane * V) % parts;
 #pragma unroll
-            for (int t = 0; t < V; ++t) {
-                const int c = lane * V + t;
-                mine |= (unsigned)(c < c_end && (lvl != 2 || (base + c) % parts == part)) << t;
+                for (int t = 0; t < V; ++t) {
+                    mine |= (unsigned)(lane * V + t < c_end && r == part) << t;
+                    r = r + 1 == parts ? 0 : r + 1;
+                }
+            } else {
+#pragma unroll
+                for (int t = 0; t < V; ++t) mine |= (unsigned)(lane * V + t < c_end) << t;
             }
             int c = F;
             if (pass1) {                                         // closest owned child (R4)
