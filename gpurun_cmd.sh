@@ -1,3 +1,6 @@
-O=gpurun_out/r02dk; mkdir -p $O
-for s in 2 4 8; do timeout 900 python bench.py --config C3 --mode data --slab $s --steps 50 --no-cpu-baseline --no-extras > $O/bench_C3_slab$s.json 2> $O/bench_C3_slab$s.err; done
-for f in $O/*.json; do echo $f; head -c 250 $f; echo; done
+O=gpurun_out/r02dp; mkdir -p $O
+for r in 1 2; do for c in C3 C4; do
+  timeout 300 python tools/var_ab.py $c psb 0 > $O/ab_base_${c}_$r.txt 2>&1
+  PSB_LIB_PATH=$PWD/paper_conf_icpp_namkn16_b200/libpsb_pp.so timeout 300 python tools/var_ab.py $c psb 0 > $O/ab_pp_${c}_$r.txt 2>&1
+done; done
+for f in $O/ab_*; do echo "$f $(tail -1 $f | cut -c1-40)"; done
